@@ -1,0 +1,183 @@
+/*
+ * emb.h -- C ABI of libemb: the B200-native PGAS-style EMB-layer forward.
+ *
+ * What it computes (PAPER.md, /root/reference/PAPER.md):
+ *   - lookup + sum pooling of embedding rows per (table, sample) bag
+ *     (L91-95, §II-B, Fig. 3);
+ *   - table-wise model parallelism with the batch-sharded data-parallel output
+ *     layout (L99-113, §II-C, Fig. 4): rank r ends with Y_r[B_r][T][d], the pooled
+ *     vectors of ALL T tables for its contiguous mini-batch;
+ *   - the paper's PGAS fused retrieval (L129-147, §III-B/C, Listing 2):
+ *     each pooled vector is stored by the kernel straight into its final slot of
+ *     the owning rank's output (one-sided peer stores over NVLink), replacing the
+ *     NCCL all-to-all + unpack of the baseline (L155, L193, §IV);
+ *   - the conventional comparison path's two kernels (pool into a send buffer,
+ *     unpack the received buffer); the all-to-all between them is NCCL, called by
+ *     the caller (PyTorch) -- L155/L193.
+ *
+ * The paper's user-facing call is forward(weights, offsets, indices, outputs)
+ * (Listing 1; Listing 2).  This ABI keeps those four
+ * roles per rank process and stream-ordered; output storage is library-owned
+ * (symmetric across ranks, PGAS style, L216/L228/L232).
+ *
+ * Conventions
+ *   - One context per rank process (or per simulated rank, see emb_init).  All
+ *     calls on a context come from one host thread.  No C++ exception crosses the
+ *     ABI; every call returns an emb_status_t and, on failure, a message is kept
+ *     for emb_last_error().
+ *   - "stream" arguments are cudaStream_t handles passed as void* (NULL = legacy
+ *     default stream).  All device work is stream-ordered and asynchronous.
+ *   - Device pointers are plain CUDA device addresses of the context's device.
+ *   - Collective calls (emb_register_tables, emb_forward, emb_finalize) must be
+ *     entered by every rank, in the same order.
+ *   - Readings of points the paper leaves open are listed in DESIGN.md (C1..C29).
+ */
+#ifndef EMB_H_
+#define EMB_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct emb_ctx emb_ctx_t;
+
+typedef enum {
+  EMB_OK = 0,
+  EMB_ERR_ARG = 1,      /* invalid argument (message in emb_last_error)            */
+  EMB_ERR_STATE = 2,    /* call out of order (e.g. forward before register)        */
+  EMB_ERR_CUDA = 3,     /* a CUDA runtime call failed                              */
+  EMB_ERR_NOMEM = 4,    /* device or host allocation failed                        */
+  EMB_ERR_PEER = 5,     /* peer exchange / IPC mapping failed                      */
+  EMB_ERR_TIMEOUT = 6,  /* a device-side peer wait timed out (see device error)    */
+  EMB_ERR_BOUNDS = 7    /* an out-of-range index was seen under CHECK_BOUNDS       */
+} emb_status_t;
+
+typedef enum { EMB_F32 = 0, EMB_BF16 = 1 } emb_dtype_t;
+
+/* emb_forward / emb_baseline_pool flags */
+#define EMB_FWD_CHECK_BOUNDS 0x1u  /* skip indices outside [0, rows) and set EMB_DEVERR_BOUNDS */
+#define EMB_FWD_SEPARATE_WAIT 0x2u /* fused kernel only signals; call emb_wait() to complete  */
+
+/* sticky device error word bits (emb_query_device_error) */
+#define EMB_DEVERR_TIMEOUT 0x1u
+#define EMB_DEVERR_BOUNDS 0x2u
+
+/* All-gather over the caller's process group.  send: `bytes` bytes of this rank;
+ * recv: world_size*bytes, rank order.  Return 0 on success.  Called only from
+ * emb_register_tables and emb_finalize (once each, plus a barrier-style call). */
+typedef int (*emb_allgather_fn)(void* user, const void* send, void* recv, size_t bytes);
+
+typedef struct {
+  int32_t rank, world_size, device, num_sms;
+  int32_t num_tables;         /* T (global)                                   */
+  int32_t num_local_tables;   /* T_r                                          */
+  int32_t dim;                /* d                                            */
+  int32_t weight_dtype, out_dtype;
+  int64_t global_batch;       /* B                                            */
+  int64_t local_batch_start;  /* s_r                                          */
+  int64_t local_batch;        /* B_r                                          */
+  uint64_t epoch;             /* number of emb_forward calls so far           */
+  int32_t grid, block;        /* fused kernel launch shape                    */
+  int32_t lanes, vec_bytes, vecs_per_lane; /* row-gather tiling                */
+  int64_t out_slot_bytes;     /* B_r*T*d*e_o                                  */
+} emb_info_t;
+
+/* Create a context for `rank` of `world_size` on CUDA device `cuda_device`.
+ * `allgather` (+ opaque `user`) is the process-group all-gather used to exchange
+ * the 64-byte CUDA IPC handles of the symmetric output buffers (may be NULL
+ * only when world_size == 1).  Several contexts may live in one process
+ * (single-process simulation of G ranks): peers in the same process are mapped
+ * by raw pointer instead of IPC.  Errors: EMB_ERR_ARG, EMB_ERR_CUDA, EMB_ERR_NOMEM. */
+emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_fn allgather, void* user,
+                      emb_ctx_t** out);
+
+/* Collective.  Describe ALL T tables and register this rank's local ones.
+ *   rows[T]    : rows M_t of every table (host)
+ *   owner[T]   : rank holding table t, in [0, world_size) (host)  -- table-wise MP (L99-101)
+ *   dim        : embedding dim d; d*sizeof(weight) must be a multiple of 8 and either
+ *                <= 512 bytes or a multiple of 512 bytes up to 4096
+ *   weight_dtype / out_dtype : EMB_F32 or EMB_BF16 (accumulation is always fp32, C5;
+ *                bf16 output is RNE-rounded once, C6)
+ *   global_batch: B >= world_size; rank r's mini-batch is the contiguous block
+ *                [s_r, s_r + B_r), first B mod G ranks one extra sample (C8)
+ *   local_weights[T_r] : device pointers of this rank's tables in ascending global id,
+ *                row-major [M_t][d], 16-byte aligned; zero-copy: the caller keeps them
+ *                alive until emb_finalize.
+ * Allocates the symmetric output (2 slots of [B_r][T][d]) + flag words, exchanges IPC
+ * handles through `allgather`, maps every peer.  Errors: EMB_ERR_ARG, EMB_ERR_STATE
+ * (already registered), EMB_ERR_CUDA/NOMEM, EMB_ERR_PEER. */
+emb_status_t emb_register_tables(emb_ctx_t* ctx, int32_t num_tables, const int64_t* rows, const int32_t* owner,
+                                 int32_t dim, emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
+                                 const void* const* local_weights);
+
+/* Collective, stream-ordered, asynchronous: the fused PGAS forward (Listing 2).
+ *   offsets : device int64[T_r*B + 1], table-major CSR: bag (t_l, b) spans
+ *             indices[offsets[t_l*B+b] .. offsets[t_l*B+b+1]) (C11; L212-215)
+ *   indices : device int64 local row ids in [0, M_t) (C1, C12)
+ *   *out    : receives the device pointer of Y_r = [B_r][T][d] (out dtype) for this
+ *             epoch; library-owned, valid until the 2nd subsequent emb_forward or
+ *             emb_finalize.  The output of epoch e must be consumed on `stream`
+ *             (or a stream ordered after it) before this rank's forward e+2.
+ * Without EMB_FWD_SEPARATE_WAIT the kernel completes only when every peer's
+ * pooled vectors for this rank have landed (in-kernel acquire wait), so any later
+ * work on `stream` sees the whole Y_r.  Empty bags produce +0.0 (C2).
+ * Errors: EMB_ERR_STATE (not registered), EMB_ERR_ARG, EMB_ERR_CUDA.  Device-side
+ * failures (peer timeout, bounds) set the sticky device error word instead. */
+emb_status_t emb_forward(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, uint32_t flags,
+                         void* stream, void** out);
+
+/* Complete a forward issued with EMB_FWD_SEPARATE_WAIT: enqueue the acquire wait on
+ * every peer's flag for the latest epoch on `stream`. */
+emb_status_t emb_wait(emb_ctx_t* ctx, void* stream);
+
+/* End-to-end convenience: host CSR in, host Y_r out (e2e measurement).  Copies
+ * h_offsets[T_r*B+1] and h_indices[h_offsets[T_r*B]] into library-owned device
+ * staging (grown on demand), runs emb_forward, copies Y_r into h_out
+ * (B_r*T*d*e_o bytes).  Host buffers should be pinned for asynchrony; the caller
+ * synchronizes `stream` before reading h_out. */
+emb_status_t emb_forward_host(emb_ctx_t* ctx, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
+                              void* stream, void* h_out);
+
+/* Collective: waits for the device, unmaps peers, frees everything, destroys ctx. */
+emb_status_t emb_finalize(emb_ctx_t* ctx);
+
+/* Mini-batch [*start, *start + *count) of `rank` (C8). */
+emb_status_t emb_local_batch(const emb_ctx_t* ctx, int rank, int64_t* start, int64_t* count);
+
+emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
+
+/* Tunables (take effect on the next launch): "chunk_rows" (target rows per claimed
+ * work chunk, default 256), "ctas_per_sm" (0 = occupancy max), "stagger" (1 =
+ * destination-staggered chunk order, default), "timeout_ms" (peer wait, default
+ * 10000 or env EMB_TIMEOUT_MS), "unroll" (rows in flight per warp: 4, 8 or 16). */
+emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
+
+/* Read (after synchronizing the forward's stream) and optionally clear the sticky
+ * device error word (EMB_DEVERR_* bits). */
+emb_status_t emb_query_device_error(emb_ctx_t* ctx, uint32_t* word, int clear);
+
+/* Last error message of this context (or of the last failed emb_init when ctx is NULL). */
+const char* emb_last_error(const emb_ctx_t* ctx);
+
+/* ---- comparison path (L155, L193) -------------------------------
+ * Split sizes (in ELEMENTS of out dtype) for torch.distributed.all_to_all_single:
+ * send_counts[dst] = B_dst*T_r*d, recv_counts[src] = B_r*T_src*d. */
+emb_status_t emb_baseline_splits(const emb_ctx_t* ctx, int64_t* send_counts, int64_t* recv_counts);
+
+/* Same gather+pool core as emb_forward, written destination-major into the
+ * caller-owned device buffer send = [G][B_dst][T_r][d] (out dtype). */
+emb_status_t emb_baseline_pool(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, uint32_t flags,
+                               void* stream, void* send);
+
+/* Unpack/rearrange after the all-to-all: recv = [G][B_r][T_src][d] (blocks in
+ * source-rank order, tables of each source in ascending global id) into
+ * out = [B_r][T][d] (caller-owned device buffers, out dtype). */
+emb_status_t emb_baseline_unpack(emb_ctx_t* ctx, const void* recv, void* stream, void* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EMB_H_ */

@@ -1,0 +1,581 @@
+// emb_runtime.cu -- the C ABI of include/emb.h: context, validation, symmetric output
+// allocator with CUDA-IPC peer mapping, epochs, launches.
+//
+// PAPER.md passages: the host side of Listing 2 (L235-254: PGAS_EMB_forward launches
+// the fused kernel per device on a non-blocking stream, then synchronizes) becomes
+// one context per rank process, launching on the caller's stream; the paper's
+// symmetric `outputs` array addressed on any PE (L216, L228, L232) becomes a
+// cudaMalloc'd buffer per rank whose IPC handle is all-gathered once over the
+// caller's process group.
+#include <cuda_runtime.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/emb.h"
+#include "emb_kernels.cuh"
+
+using namespace emb;
+
+namespace {
+
+constexpr uint64_t kMagic = 0x454d42504741531full;  // "EMBPGAS"
+
+struct PeerBlob {
+  uint64_t magic;
+  int32_t rank, pid;
+  uint64_t host_hash;
+  uint64_t ptr;          // base of the symmetric allocation in the owner's process
+  uint64_t bytes;
+  uint64_t slot_off;     // byte offset of slot 0
+  uint64_t slot_bytes;   // bytes per slot (B_r*T*d*e_o rounded up to 256)
+  int32_t device;
+  int32_t pad;
+  cudaIpcMemHandle_t handle;
+};
+
+std::string g_init_error;
+
+uint64_t host_hash() {
+  char name[256] = {0};
+  gethostname(name, sizeof(name) - 1);
+  uint64_t h = 1469598103934665603ull;
+  for (const char* c = name; *c; ++c) h = (h ^ (uint64_t)(unsigned char)*c) * 1099511628211ull;
+  return h;
+}
+
+size_t round_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+}  // namespace
+
+struct emb_ctx {
+  int rank = 0, G = 1, dev = 0, num_sms = 148;
+  emb_allgather_fn ag = nullptr;
+  void* user = nullptr;
+  bool registered = false;
+  // tables
+  int T = 0, T_r = 0, d = 0;
+  emb_dtype_t wdt = EMB_F32, odt = EMB_F32;
+  int64_t B = 0;
+  std::vector<int64_t> rows;
+  std::vector<int32_t> owner;
+  std::vector<int64_t> bstart;          // G+1
+  std::vector<int32_t> local;           // global ids of local tables
+  std::vector<int32_t> tables_of[kMaxG];
+  TableDesc* d_tables = nullptr;
+  // symmetric buffer (flags at offset 0, slots after)
+  char* sym = nullptr;
+  size_t sym_bytes = 0, slot_off = 0, slot_bytes = 0;
+  std::vector<char*> peer_base;         // mapped base per rank
+  std::vector<uint64_t> peer_slot_off, peer_slot_bytes;
+  std::vector<bool> peer_ipc;           // opened through cudaIpcOpenMemHandle
+  Ctrl* ctrl = nullptr;
+  uint64_t epoch = 0;
+  // options
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 8;
+  int64_t timeout_ns = 10000000000ll;
+  // gather tiling
+  int lanes = 32, vb = 16, nv = 1;
+  // comparison path
+  int64_t* d_unpack_base = nullptr;
+  int32_t* d_unpack_stride = nullptr;
+  // e2e staging
+  int64_t* d_off_stage = nullptr;
+  int64_t* d_idx_stage = nullptr;
+  size_t idx_cap = 0;
+  std::string err;
+  FwdParams last{};
+};
+
+#define FAIL(ctx, code, ...)                        \
+  do {                                              \
+    char _b[512];                                   \
+    snprintf(_b, sizeof(_b), __VA_ARGS__);          \
+    if (ctx) (ctx)->err = _b; else g_init_error = _b; \
+    return code;                                    \
+  } while (0)
+
+#define CK(ctx, call)                                                                                   \
+  do {                                                                                                  \
+    cudaError_t _e = (call);                                                                            \
+    if (_e != cudaSuccess) FAIL(ctx, EMB_ERR_CUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(_e), \
+                                __FILE__, __LINE__);                                                    \
+  } while (0)
+
+static size_t esize(emb_dtype_t t) { return t == EMB_F32 ? 4 : 2; }
+
+// ---------------------------------------------------------------------------- kernel dispatch
+namespace {
+
+using KernelFn = void (*)(FwdParams);
+
+template <int VB, int NV, typename WT, typename OT>
+KernelFn pick_u(int unroll, bool check) {
+  switch (unroll) {
+    case 4:
+      return check ? emb_fwd_kernel<VB, NV, WT, OT, 4, true> : emb_fwd_kernel<VB, NV, WT, OT, 4, false>;
+    case 16:
+      return check ? emb_fwd_kernel<VB, NV, WT, OT, 16, true> : emb_fwd_kernel<VB, NV, WT, OT, 16, false>;
+    default:
+      return check ? emb_fwd_kernel<VB, NV, WT, OT, 8, true> : emb_fwd_kernel<VB, NV, WT, OT, 8, false>;
+  }
+}
+
+template <typename WT, typename OT>
+KernelFn pick_tile(int vb, int nv, int unroll, bool check) {
+  if (vb == 8) return pick_u<8, 1, WT, OT>(unroll, check);
+  switch (nv) {
+    case 2: return pick_u<16, 2, WT, OT>(unroll, check);
+    case 4: return pick_u<16, 4, WT, OT>(unroll, check);
+    case 8: return pick_u<16, 8, WT, OT>(unroll, check);
+    default: return pick_u<16, 1, WT, OT>(unroll, check);
+  }
+}
+
+KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check) {
+  if (w == EMB_F32 && o == EMB_F32) return pick_tile<float, float>(vb, nv, unroll, check);
+  if (w == EMB_F32 && o == EMB_BF16) return pick_tile<float, __nv_bfloat16>(vb, nv, unroll, check);
+  if (w == EMB_BF16 && o == EMB_F32) return pick_tile<__nv_bfloat16, float>(vb, nv, unroll, check);
+  return pick_tile<__nv_bfloat16, __nv_bfloat16>(vb, nv, unroll, check);
+}
+
+// row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
+bool choose_tiling(int64_t rowbytes, size_t wsz, size_t osz, int* lanes, int* vb, int* nv) {
+  if (rowbytes <= 0) return false;
+  if (rowbytes == 256) { *vb = 8; *nv = 1; *lanes = 32; }
+  else if (rowbytes % 16 == 0 && rowbytes <= 512) { *vb = 16; *nv = 1; *lanes = (int)(rowbytes / 16); }
+  else if (rowbytes % 512 == 0 && rowbytes <= 4096 && (rowbytes / 512 == 2 || rowbytes / 512 == 4 || rowbytes / 512 == 8)) {
+    *vb = 16; *nv = (int)(rowbytes / 512); *lanes = 32;
+  } else if (rowbytes % 8 == 0 && rowbytes < 256) { *vb = 8; *nv = 1; *lanes = (int)(rowbytes / 8); }
+  else return false;
+  // output vector per lane must be >= 4 bytes
+  const int epv = *vb / (int)wsz;
+  return epv * (int)osz >= 4;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------- API
+extern "C" {
+
+emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_fn allgather, void* user,
+                      emb_ctx_t** out) {
+  if (!out) FAIL((emb_ctx_t*)nullptr, EMB_ERR_ARG, "out is NULL");
+  *out = nullptr;
+  if (world_size < 1 || world_size > kMaxG) FAIL((emb_ctx_t*)nullptr, EMB_ERR_ARG, "world_size %d not in [1, %d]", world_size, kMaxG);
+  if (rank < 0 || rank >= world_size) FAIL((emb_ctx_t*)nullptr, EMB_ERR_ARG, "rank %d not in [0, %d)", rank, world_size);
+  if (world_size > 1 && !allgather) FAIL((emb_ctx_t*)nullptr, EMB_ERR_ARG, "allgather callback required for world_size > 1");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0)
+    FAIL((emb_ctx_t*)nullptr, EMB_ERR_CUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  if (cuda_device < 0 || cuda_device >= ndev) FAIL((emb_ctx_t*)nullptr, EMB_ERR_ARG, "cuda_device %d not in [0, %d)", cuda_device, ndev);
+  emb_ctx_t* c = new (std::nothrow) emb_ctx_t();
+  if (!c) FAIL((emb_ctx_t*)nullptr, EMB_ERR_NOMEM, "host allocation failed");
+  c->rank = rank;
+  c->G = world_size;
+  c->dev = cuda_device;
+  c->ag = allgather;
+  c->user = user;
+  if (const char* s = getenv("EMB_TIMEOUT_MS")) c->timeout_ns = atoll(s) * 1000000ll;
+  e = cudaSetDevice(cuda_device);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  if (e == cudaSuccess) e = cudaMalloc(&c->ctrl, sizeof(Ctrl));
+  if (e == cudaSuccess) e = cudaMemset(c->ctrl, 0, sizeof(Ctrl));
+  if (e != cudaSuccess) {
+    g_init_error = std::string("CUDA init failed: ") + cudaGetErrorString(e);
+    delete c;
+    return EMB_ERR_CUDA;
+  }
+  *out = c;
+  return EMB_OK;
+}
+
+emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t* rows, const int32_t* owner,
+                                 int32_t dim, emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
+                                 const void* const* local_weights) {
+  if (!c) return EMB_ERR_ARG;
+  if (c->registered) FAIL(c, EMB_ERR_STATE, "tables already registered");
+  if (num_tables < 1 || !rows || !owner) FAIL(c, EMB_ERR_ARG, "num_tables/rows/owner invalid");
+  if (weight_dtype != EMB_F32 && weight_dtype != EMB_BF16) FAIL(c, EMB_ERR_ARG, "bad weight dtype");
+  if (out_dtype != EMB_F32 && out_dtype != EMB_BF16) FAIL(c, EMB_ERR_ARG, "bad out dtype");
+  if (global_batch < c->G) FAIL(c, EMB_ERR_ARG, "global_batch %lld < world_size %d", (long long)global_batch, c->G);
+  if (dim < 1) FAIL(c, EMB_ERR_ARG, "dim %d < 1", dim);
+  const size_t wsz = esize(weight_dtype), osz = esize(out_dtype);
+  int lanes, vb, nv;
+  if (!choose_tiling((int64_t)dim * wsz, wsz, osz, &lanes, &vb, &nv))
+    FAIL(c, EMB_ERR_ARG, "unsupported row size d*e = %lld bytes (need multiple of 8, <= 512 or 1024/2048/4096)",
+         (long long)dim * (long long)wsz);
+  if (((int64_t)dim * (int64_t)osz) % 16 != 0 && c->G > 1) {
+    // unpack kernel moves 8-byte pieces at least
+    if (((int64_t)dim * (int64_t)osz) % 8 != 0) FAIL(c, EMB_ERR_ARG, "output row bytes must be a multiple of 8");
+  }
+  c->T = num_tables;
+  c->d = dim;
+  c->wdt = weight_dtype;
+  c->odt = out_dtype;
+  c->B = global_batch;
+  c->lanes = lanes;
+  c->vb = vb;
+  c->nv = nv;
+  c->rows.assign(rows, rows + num_tables);
+  c->owner.assign(owner, owner + num_tables);
+  c->local.clear();
+  for (int g = 0; g < kMaxG; ++g) c->tables_of[g].clear();
+  for (int t = 0; t < num_tables; ++t) {
+    if (rows[t] < 1) FAIL(c, EMB_ERR_ARG, "rows[%d] = %lld < 1", t, (long long)rows[t]);
+    if (owner[t] < 0 || owner[t] >= c->G) FAIL(c, EMB_ERR_ARG, "owner[%d] = %d not in [0, %d)", t, owner[t], c->G);
+    c->tables_of[owner[t]].push_back(t);
+    if (owner[t] == c->rank) c->local.push_back(t);
+  }
+  c->T_r = (int)c->local.size();
+  // contiguous batch split (C8)
+  c->bstart.assign(c->G + 1, 0);
+  {
+    const int64_t q = global_batch / c->G, rem = global_batch % c->G;
+    for (int r = 0; r < c->G; ++r) c->bstart[r + 1] = c->bstart[r] + q + (r < rem ? 1 : 0);
+  }
+  CK(c, cudaSetDevice(c->dev));
+  // table descriptors
+  std::vector<TableDesc> td(std::max(c->T_r, 1));
+  for (int i = 0; i < c->T_r; ++i) {
+    const void* w = local_weights ? local_weights[i] : nullptr;
+    if (!w) FAIL(c, EMB_ERR_ARG, "local_weights[%d] is NULL", i);
+    if (((uintptr_t)w) % 16 != 0) FAIL(c, EMB_ERR_ARG, "local_weights[%d] not 16-byte aligned", i);
+    td[i].w = w;
+    td[i].rows = rows[c->local[i]];
+    td[i].tglob = c->local[i];
+    td[i].pad = 0;
+  }
+  CK(c, cudaMalloc(&c->d_tables, td.size() * sizeof(TableDesc)));
+  CK(c, cudaMemcpy(c->d_tables, td.data(), td.size() * sizeof(TableDesc), cudaMemcpyHostToDevice));
+  // unpack maps: recv = [G][B_r][T_src][d]; vector index of (b, t) = R0[src] + b*T_src + t_l
+  {
+    const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+    std::vector<int64_t> base(num_tables);
+    std::vector<int32_t> stride(num_tables);
+    int64_t R0 = 0;
+    for (int s = 0; s < c->G; ++s) {
+      const int Ts = (int)c->tables_of[s].size();
+      for (int i = 0; i < Ts; ++i) {
+        base[c->tables_of[s][i]] = R0 + i;
+        stride[c->tables_of[s][i]] = Ts;
+      }
+      R0 += Br * Ts;
+    }
+    CK(c, cudaMalloc(&c->d_unpack_base, num_tables * sizeof(int64_t)));
+    CK(c, cudaMalloc(&c->d_unpack_stride, num_tables * sizeof(int32_t)));
+    CK(c, cudaMemcpy(c->d_unpack_base, base.data(), num_tables * sizeof(int64_t), cudaMemcpyHostToDevice));
+    CK(c, cudaMemcpy(c->d_unpack_stride, stride.data(), num_tables * sizeof(int32_t), cudaMemcpyHostToDevice));
+  }
+  // symmetric buffer: [flags: G u32, padded to 512 B][slot 0][slot 1]
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  c->slot_off = 512;
+  c->slot_bytes = round_up((size_t)Br * (size_t)num_tables * (size_t)dim * osz, 512);
+  c->sym_bytes = c->slot_off + 2 * c->slot_bytes;
+  {
+    cudaError_t e = cudaMalloc(&c->sym, c->sym_bytes);
+    if (e == cudaErrorMemoryAllocation) FAIL(c, EMB_ERR_NOMEM, "symmetric buffer of %zu bytes: out of memory", c->sym_bytes);
+    CK(c, e);
+  }
+  CK(c, cudaMemset(c->sym, 0, c->slot_off));
+  // exchange
+  PeerBlob mine{};
+  mine.magic = kMagic;
+  mine.rank = c->rank;
+  mine.pid = (int32_t)getpid();
+  mine.host_hash = host_hash();
+  mine.ptr = (uint64_t)(uintptr_t)c->sym;
+  mine.bytes = c->sym_bytes;
+  mine.slot_off = c->slot_off;
+  mine.slot_bytes = c->slot_bytes;
+  mine.device = c->dev;
+  CK(c, cudaIpcGetMemHandle(&mine.handle, c->sym));
+  std::vector<PeerBlob> all(c->G);
+  if (c->G == 1) {
+    all[0] = mine;
+  } else {
+    if (c->ag(c->user, &mine, all.data(), sizeof(PeerBlob)) != 0) FAIL(c, EMB_ERR_PEER, "allgather of IPC handles failed");
+  }
+  c->peer_base.assign(c->G, nullptr);
+  c->peer_slot_off.assign(c->G, 0);
+  c->peer_slot_bytes.assign(c->G, 0);
+  c->peer_ipc.assign(c->G, false);
+  for (int p = 0; p < c->G; ++p) {
+    const PeerBlob& b = all[p];
+    if (b.magic != kMagic || b.rank != p) FAIL(c, EMB_ERR_PEER, "bad peer blob from rank %d", p);
+    if (b.host_hash != mine.host_hash) FAIL(c, EMB_ERR_PEER, "rank %d is on another host (multi-node is out of scope)", p);
+    c->peer_slot_off[p] = b.slot_off;
+    c->peer_slot_bytes[p] = b.slot_bytes;
+    if (p == c->rank) {
+      c->peer_base[p] = c->sym;
+    } else if (b.pid == mine.pid) {  // simulated rank in this process: raw pointer
+      if (b.device != c->dev) {
+        cudaError_t e = cudaDeviceEnablePeerAccess(b.device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(c, e);
+        cudaGetLastError();
+      }
+      c->peer_base[p] = (char*)(uintptr_t)b.ptr;
+    } else {
+      void* ptr = nullptr;
+      cudaError_t e = cudaIpcOpenMemHandle(&ptr, b.handle, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) FAIL(c, EMB_ERR_PEER, "cudaIpcOpenMemHandle(rank %d) failed: %s", p, cudaGetErrorString(e));
+      c->peer_base[p] = (char*)ptr;
+      c->peer_ipc[p] = true;
+    }
+  }
+  // barrier: every rank mapped everything before anyone writes
+  if (c->G > 1) {
+    int one = 1;
+    std::vector<int> r(c->G);
+    if (c->ag(c->user, &one, r.data(), sizeof(int)) != 0) FAIL(c, EMB_ERR_PEER, "registration barrier failed");
+  }
+  c->registered = true;
+  return EMB_OK;
+}
+
+static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, bool pgas, char* send,
+                                FwdParams* p) {
+  memset(p, 0, sizeof(*p));
+  p->tables = c->d_tables;
+  p->offsets = offsets;
+  p->indices = indices;
+  p->B = c->B;
+  p->T_r = c->T_r;
+  p->d = c->d;
+  p->G = c->G;
+  p->rank = c->rank;
+  p->lanes = c->lanes;
+  p->chunk_rows = c->chunk_rows;
+  p->stagger = c->stagger;
+  p->ctrl = c->ctrl;
+  p->timeout_ns = c->timeout_ns;
+  for (int g = 0; g <= c->G; ++g) p->bstart[g] = c->bstart[g];
+  for (int g = c->G + 1; g <= kMaxG; ++g) p->bstart[g] = INT64_MAX;
+  p->my_flags = reinterpret_cast<const uint32_t*>(c->sym);
+  const size_t osz = esize(c->odt);
+  if (pgas) {
+    const int slot = (int)(c->epoch & 1);  // epoch already advanced for this forward
+    p->rowstride = c->T;
+    p->use_tglob = 1;
+    p->signal = 1;
+    for (int g = 0; g < c->G; ++g) {
+      p->out_base[g] = c->peer_base[g] + c->peer_slot_off[g] + (size_t)slot * c->peer_slot_bytes[g];
+      p->peer_flag[g] = (g == c->rank) ? nullptr : reinterpret_cast<uint32_t*>(c->peer_base[g]) + c->rank;
+    }
+  } else {
+    p->rowstride = c->T_r;
+    p->use_tglob = 0;
+    p->signal = 0;
+    for (int g = 0; g < c->G; ++g)  // send = [G][B_dst][T_r][d]: block of dst starts at s_dst*T_r rows
+      p->out_base[g] = send + (size_t)c->bstart[g] * (size_t)c->T_r * (size_t)c->d * osz;
+  }
+  p->epoch = (uint32_t)c->epoch;
+  return EMB_OK;
+}
+
+static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, c->unroll, (flags & EMB_FWD_CHECK_BOUNDS) != 0);
+  int per_sm = c->ctas_per_sm;
+  if (per_sm <= 0) {
+    CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0));
+    if (per_sm < 1) per_sm = 1;
+  }
+  const int grid = c->num_sms * per_sm;
+  k<<<grid, kBlock, 0, s>>>(p);
+  CK(c, cudaGetLastError());
+  return EMB_OK;
+}
+
+emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags, void* stream,
+                         void** out) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward before emb_register_tables");
+  if (c->T_r > 0 && (!offsets || !indices)) FAIL(c, EMB_ERR_ARG, "offsets/indices NULL");
+  CK(c, cudaSetDevice(c->dev));
+  c->epoch += 1;
+  FwdParams p;
+  fill_params(c, offsets, indices, true, nullptr, &p);
+  p.wait = (flags & EMB_FWD_SEPARATE_WAIT) ? 0 : 1;
+  c->last = p;
+  emb_status_t st = launch_fwd(c, p, flags, (cudaStream_t)stream);
+  if (st != EMB_OK) return st;
+  if (out) *out = c->sym + c->slot_off + (size_t)(c->epoch & 1) * c->slot_bytes;
+  return EMB_OK;
+}
+
+emb_status_t emb_wait(emb_ctx_t* c, void* stream) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered || c->epoch == 0) FAIL(c, EMB_ERR_STATE, "emb_wait without a forward");
+  CK(c, cudaSetDevice(c->dev));
+  if (c->G == 1) return EMB_OK;
+  emb_wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(c->last);
+  CK(c, cudaGetLastError());
+  return EMB_OK;
+}
+
+emb_status_t emb_forward_host(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
+                              void* stream, void* h_out) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward_host before emb_register_tables");
+  if (!h_offsets || !h_out || (c->T_r > 0 && !h_indices)) FAIL(c, EMB_ERR_ARG, "NULL host buffer");
+  CK(c, cudaSetDevice(c->dev));
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t noff = (size_t)c->T_r * (size_t)c->B + 1;
+  const int64_t nnz = h_offsets[noff - 1];
+  if (nnz < 0) FAIL(c, EMB_ERR_ARG, "negative nnz");
+  if (!c->d_off_stage) CK(c, cudaMalloc(&c->d_off_stage, noff * sizeof(int64_t)));
+  if ((size_t)nnz > c->idx_cap || !c->d_idx_stage) {
+    CK(c, cudaStreamSynchronize(s));
+    if (c->d_idx_stage) CK(c, cudaFree(c->d_idx_stage));
+    c->idx_cap = std::max<size_t>((size_t)nnz, 1) + (size_t)nnz / 4;
+    CK(c, cudaMalloc(&c->d_idx_stage, c->idx_cap * sizeof(int64_t)));
+  }
+  CK(c, cudaMemcpyAsync(c->d_off_stage, h_offsets, noff * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+  if (nnz > 0) CK(c, cudaMemcpyAsync(c->d_idx_stage, h_indices, (size_t)nnz * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+  void* dout = nullptr;
+  emb_status_t st = emb_forward(c, c->d_off_stage, c->d_idx_stage, flags, stream, &dout);
+  if (st != EMB_OK) return st;
+  if (flags & EMB_FWD_SEPARATE_WAIT) {
+    st = emb_wait(c, stream);
+    if (st != EMB_OK) return st;
+  }
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  CK(c, cudaMemcpyAsync(h_out, dout, (size_t)Br * c->T * c->d * esize(c->odt), cudaMemcpyDeviceToHost, s));
+  return EMB_OK;
+}
+
+emb_status_t emb_finalize(emb_ctx_t* c) {
+  if (!c) return EMB_ERR_ARG;
+  cudaSetDevice(c->dev);
+  cudaDeviceSynchronize();
+  emb_status_t st = EMB_OK;
+  if (c->registered && c->G > 1) {  // nobody may still write into our buffer
+    int one = 1;
+    std::vector<int> r(c->G);
+    if (c->ag(c->user, &one, r.data(), sizeof(int)) != 0) st = EMB_ERR_PEER;
+  }
+  for (int p = 0; p < (int)c->peer_base.size(); ++p)
+    if (c->peer_ipc[p]) cudaIpcCloseMemHandle(c->peer_base[p]);
+  if (c->sym) cudaFree(c->sym);
+  if (c->d_tables) cudaFree(c->d_tables);
+  if (c->ctrl) cudaFree(c->ctrl);
+  if (c->d_unpack_base) cudaFree(c->d_unpack_base);
+  if (c->d_unpack_stride) cudaFree(c->d_unpack_stride);
+  if (c->d_off_stage) cudaFree(c->d_off_stage);
+  if (c->d_idx_stage) cudaFree(c->d_idx_stage);
+  delete c;
+  return st;
+}
+
+emb_status_t emb_local_batch(const emb_ctx_t* c, int rank, int64_t* start, int64_t* count) {
+  if (!c || !start || !count) return EMB_ERR_ARG;
+  if (!c->registered) return EMB_ERR_STATE;
+  if (rank < 0 || rank >= c->G) return EMB_ERR_ARG;
+  *start = c->bstart[rank];
+  *count = c->bstart[rank + 1] - c->bstart[rank];
+  return EMB_OK;
+}
+
+emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
+  if (!c || !i) return EMB_ERR_ARG;
+  memset(i, 0, sizeof(*i));
+  i->rank = c->rank;
+  i->world_size = c->G;
+  i->device = c->dev;
+  i->num_sms = c->num_sms;
+  i->num_tables = c->T;
+  i->num_local_tables = c->T_r;
+  i->dim = c->d;
+  i->weight_dtype = c->wdt;
+  i->out_dtype = c->odt;
+  i->global_batch = c->B;
+  if (c->registered) {
+    i->local_batch_start = c->bstart[c->rank];
+    i->local_batch = c->bstart[c->rank + 1] - c->bstart[c->rank];
+    i->out_slot_bytes = i->local_batch * c->T * c->d * (int64_t)esize(c->odt);
+  }
+  i->epoch = c->epoch;
+  int per_sm = c->ctas_per_sm;
+  if (per_sm <= 0 && c->registered) {
+    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, c->unroll, false);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0);
+  }
+  i->grid = c->num_sms * std::max(per_sm, 1);
+  i->block = kBlock;
+  i->lanes = c->lanes;
+  i->vec_bytes = c->vb;
+  i->vecs_per_lane = c->nv;
+  return EMB_OK;
+}
+
+emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
+  if (!c || !key) return EMB_ERR_ARG;
+  if (!strcmp(key, "chunk_rows")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "chunk_rows < 1"); c->chunk_rows = (int)v; }
+  else if (!strcmp(key, "ctas_per_sm")) { if (v < 0 || v > 32) FAIL(c, EMB_ERR_ARG, "ctas_per_sm"); c->ctas_per_sm = (int)v; }
+  else if (!strcmp(key, "stagger")) c->stagger = v ? 1 : 0;
+  else if (!strcmp(key, "timeout_ms")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "timeout_ms < 1"); c->timeout_ns = v * 1000000ll; }
+  else if (!strcmp(key, "unroll")) { if (v != 4 && v != 8 && v != 16) FAIL(c, EMB_ERR_ARG, "unroll must be 4, 8 or 16"); c->unroll = (int)v; }
+  else FAIL(c, EMB_ERR_ARG, "unknown option '%s'", key);
+  return EMB_OK;
+}
+
+emb_status_t emb_query_device_error(emb_ctx_t* c, uint32_t* word, int clear) {
+  if (!c || !word) return EMB_ERR_ARG;
+  CK(c, cudaSetDevice(c->dev));
+  CK(c, cudaMemcpy(word, &c->ctrl->err, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  if (clear) CK(c, cudaMemset(&c->ctrl->err, 0, sizeof(uint32_t)));
+  return EMB_OK;
+}
+
+const char* emb_last_error(const emb_ctx_t* c) { return c ? c->err.c_str() : g_init_error.c_str(); }
+
+emb_status_t emb_baseline_splits(const emb_ctx_t* c, int64_t* send_counts, int64_t* recv_counts) {
+  if (!c || !send_counts || !recv_counts) return EMB_ERR_ARG;
+  if (!c->registered) return EMB_ERR_STATE;
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  for (int g = 0; g < c->G; ++g) {
+    send_counts[g] = (c->bstart[g + 1] - c->bstart[g]) * c->T_r * c->d;
+    recv_counts[g] = Br * (int64_t)c->tables_of[g].size() * c->d;
+  }
+  return EMB_OK;
+}
+
+emb_status_t emb_baseline_pool(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags,
+                               void* stream, void* send) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_pool before emb_register_tables");
+  if (c->T_r > 0 && (!offsets || !indices || !send)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
+  CK(c, cudaSetDevice(c->dev));
+  FwdParams p;
+  fill_params(c, offsets, indices, false, (char*)send, &p);
+  return launch_fwd(c, p, flags & EMB_FWD_CHECK_BOUNDS, (cudaStream_t)stream);
+}
+
+emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, void* out) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_unpack before emb_register_tables");
+  if (!recv || !out) FAIL(c, EMB_ERR_ARG, "NULL buffer");
+  CK(c, cudaSetDevice(c->dev));
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  const int rowbytes = c->d * (int)esize(c->odt);
+  const int64_t pieces = Br * c->T * (rowbytes % 16 == 0 ? rowbytes / 16 : rowbytes / 8);
+  int grid = (int)std::min<int64_t>((pieces + kBlock - 1) / kBlock, (int64_t)c->num_sms * 8);
+  if (grid < 1) grid = 1;
+  if (rowbytes % 16 == 0)
+    emb_unpack_kernel<<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out, c->d_unpack_base,
+                                                                  c->d_unpack_stride, Br, c->T, rowbytes);
+  else
+    emb_unpack8_kernel<<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out, c->d_unpack_base,
+                                                                   c->d_unpack_stride, Br, c->T, rowbytes);
+  CK(c, cudaGetLastError());
+  return EMB_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,93 @@
+"""Rank-level EMB layer on top of the C ABI (Listing 1: the DLRM
+calls LookupFunction.apply(weights, offsets, indices, outputs) and continues with
+`outputs`).  Holds the context, exposes the PGAS forward and the conventional
+comparison path (pool kernel -> NCCL all_to_all_single -> unpack kernel, L155/L193).
+Marshalling only: all arithmetic runs in libemb.so.
+"""
+from __future__ import annotations
+
+from typing import Optional, Sequence
+
+import torch
+
+from . import emb as E
+
+
+class _CAI:
+    def __init__(self, ptr: int, shape, typestr: str):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr, "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
+def wrap_device(ptr: int, shape, dtype: torch.dtype, device) -> torch.Tensor:
+    """Zero-copy torch view of a library-owned device buffer."""
+    if dtype == torch.float32:
+        return torch.as_tensor(_CAI(ptr, shape, "<f4"), device=device)
+    if dtype == torch.bfloat16:
+        return torch.as_tensor(_CAI(ptr, shape, "<i2"), device=device).view(torch.bfloat16)
+    raise ValueError(dtype)
+
+
+def _tdt(code: int) -> torch.dtype:
+    return torch.float32 if code == E.EMB_F32 else torch.bfloat16
+
+
+class PgasEmbedding:
+    """One rank's share of a table-wise model-parallel EMB layer."""
+
+    def __init__(self, rank: int, world_size: int, device: int, rows: Sequence[int], owner: Sequence[int], dim: int,
+                 local_weights: Sequence[torch.Tensor], global_batch: int, weight_dtype="f32", out_dtype="f32",
+                 allgather=None, options: Optional[dict] = None):
+        self.device = torch.device("cuda", device)
+        self.ctx = E.emb_init(rank, world_size, device, allgather)
+        self._weights = list(local_weights)  # zero-copy: keep alive
+        E.emb_register_tables(self.ctx, rows, owner, dim, weight_dtype, out_dtype, global_batch, self._weights)
+        for k, v in (options or {}).items():
+            E.emb_set_option(self.ctx, k, v)
+        self.info = E.emb_get_info(self.ctx)
+        self.T = self.info["num_tables"]
+        self.T_r = self.info["num_local_tables"]
+        self.dim = dim
+        self.B = global_batch
+        self.B_r = self.info["local_batch"]
+        self.out_dtype = _tdt(self.info["out_dtype"])
+        self._send = self._recv = self._out = None
+
+    # ---- PGAS fused path (Listing 2) ----------------------------------------------------
+    def forward(self, offsets: torch.Tensor, indices: torch.Tensor, flags: int = 0, stream=None) -> torch.Tensor:
+        ptr = E.emb_forward(self.ctx, offsets, indices, flags, stream)
+        return wrap_device(ptr, (self.B_r, self.T, self.dim), self.out_dtype, self.device)
+
+    def wait(self, stream=None) -> None:
+        E.emb_wait(self.ctx, stream)
+
+    # ---- comparison path (L155, L193) ---------------------------------------------------
+    def _baseline_buffers(self):
+        if self._send is None:
+            sc, rc = E.emb_baseline_splits(self.ctx)
+            self._send_counts, self._recv_counts = sc, rc
+            self._send = torch.empty(max(sum(sc), 1), dtype=self.out_dtype, device=self.device)
+            self._recv = torch.empty(max(sum(rc), 1), dtype=self.out_dtype, device=self.device)
+            self._out = torch.empty((self.B_r, self.T, self.dim), dtype=self.out_dtype, device=self.device)
+        return self._send, self._recv, self._out
+
+    def forward_baseline(self, offsets: torch.Tensor, indices: torch.Tensor, group=None, flags: int = 0,
+                         stream=None) -> torch.Tensor:
+        send, recv, out = self._baseline_buffers()
+        E.emb_baseline_pool(self.ctx, offsets, indices, send, flags, stream)
+        if self.ctx.world_size == 1:  # G = 1: send already is [B][T][d]; no exchange, no unpack
+            return send[: self.B_r * self.T * self.dim].view(self.B_r, self.T, self.dim)
+        import torch.distributed as dist
+        work = dist.all_to_all_single(recv, send, output_split_sizes=self._recv_counts,
+                                      input_split_sizes=self._send_counts, group=group, async_op=True)
+        work.wait()
+        E.emb_baseline_unpack(self.ctx, recv, out, stream)
+        return out
+
+    def device_error(self, clear: bool = False) -> int:
+        return E.emb_query_device_error(self.ctx, clear)
+
+    def close(self) -> None:
+        if self.ctx is not None and self.ctx.ptr:
+            E.emb_finalize(self.ctx)
+        self.ctx = None

@@ -1,0 +1,327 @@
+"""GPU parity: libemb.so (through the C ABI) vs the CPU oracle, element by element.
+
+Bar (BASELINE.json north_star): bit-exact for placement/indices; fp32 values within
+S-normalised 1e-6, bf16 within 1e-2.  The kernel keeps the canonical CSR summation
+order (C4), so it is additionally required to be BIT-EXACT to the canonical oracle.
+"""
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import synth
+from oracle import emb_oracle as O
+import emb_test_helpers as H
+
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_sc_chenbyo24_b200 import emb as E  # noqa: E402
+from paper_conf_sc_chenbyo24_b200.comm import LocalGroup, run_ranks  # noqa: E402
+from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding  # noqa: E402
+
+DEV = torch.device("cuda", 0)
+
+
+def _dev_tables(w, tabs_np, r):
+    out = []
+    for t in w.local_tables(r):
+        a = tabs_np[int(w.phys[t])]
+        if w.wdtype == "bf16":
+            out.append(torch.from_numpy(synth.to_bf16_bits(a).view(np.int16)).to(DEV).view(torch.bfloat16))
+        else:
+            out.append(torch.from_numpy(a).to(DEV))
+    return out
+
+
+def _layers(w, tabs_np, options=None):
+    """One PgasEmbedding per simulated rank (single process, one GPU)."""
+    tabs_dev = [_dev_tables(w, tabs_np, r) for r in range(w.G)]
+    if w.G == 1:
+        return [PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, tabs_dev[0], w.B, w.wdtype, w.odtype, None, options)]
+    grp = LocalGroup(w.G)
+    return run_ranks(w.G, lambda r: PgasEmbedding(r, w.G, 0, w.rows, w.owner, w.dim, tabs_dev[r], w.B, w.wdtype,
+                                                  w.odtype, grp.allgather_for(r), options))
+
+
+def _run(w, layers, csr_np, flags=0, streams=None):
+    offs, idxs = csr_np
+    dev_in = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(w.G)]
+    streams = streams or [torch.cuda.Stream() for _ in range(w.G)]
+    torch.cuda.synchronize()
+    ys = []
+    for r in range(w.G):
+        ys.append(layers[r].forward(dev_in[r][0], dev_in[r][1], flags, streams[r]))
+    if flags & E.EMB_FWD_SEPARATE_WAIT:
+        for r in range(w.G):
+            layers[r].wait(streams[r])
+    torch.cuda.synchronize()
+    return [H.dev_out_to_np(y.clone()) for y in ys]
+
+
+def _close(layers):
+    if len(layers) == 1:
+        layers[0].close()
+    else:
+        run_ranks(len(layers), lambda r: layers[r].close())
+
+
+def _assert_exact(got, ref):
+    assert got.shape == ref.shape
+    gb, rb = H.bits(got), H.bits(ref)
+    if not np.array_equal(gb, rb):
+        bad = np.argwhere(gb != rb)
+        raise AssertionError(f"{len(bad)} mismatches, first at {bad[0].tolist()}: got {got[tuple(bad[0])]} "
+                             f"want {ref[tuple(bad[0])]}")
+
+
+# ------------------------------------------------------------------------------- G = 1
+CASES = [
+    # name, overrides
+    ("tiny", dict()),
+    ("tiny", dict(pmin=0, pmax=9, B=1000, T=5, rows=777)),          # empty bags, ragged chunks
+    ("tiny", dict(dim=64, pmin=1, pmax=128, B=300, rows=5000)),      # 256-B rows (LDG.64 path)
+    ("tiny", dict(dim=128, pmin=0, pmax=40, B=513, rows=3000, dist="zipf")),
+    ("tiny", dict(dim=256, pmin=1, pmax=20, B=257, rows=999)),       # 1-KB rows (2 vectors per lane)
+    ("tiny", dict(dim=8, pmin=1, pmax=7, B=100)),                    # 32-B rows (2 active lanes)
+    ("tiny", dict(dim=512, pmin=1, pmax=5, B=65, rows=100)),         # 2-KB rows
+    ("tiny", dict(dim=128, wdtype="bf16", odtype="bf16", pmin=1, pmax=100, B=200, rows=4000)),
+    ("tiny", dict(dim=256, wdtype="bf16", odtype="bf16", pmin=0, pmax=60, B=130, rows=4000)),
+    ("tiny", dict(dim=64, wdtype="f32", odtype="bf16", pmin=1, pmax=33, B=200)),
+    ("tiny", dict(dim=64, wdtype="bf16", odtype="f32", pmin=1, pmax=33, B=200)),
+    ("tiny", dict(dim=16, pmin=1, pmax=1, B=64, T=3)),               # one-hot bags
+]
+
+
+@pytest.mark.parametrize("name,over", CASES)
+def test_g1_bitexact_vs_oracle(name, over):
+    w = synth.make_workload(name, G=1, **over)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 101)
+    ref = H.oracle_outputs(w, 101, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, csr)
+    finally:
+        _close(layers)
+    _assert_exact(got[0], ref[0])
+
+
+def test_integer_tables_exact_and_tolerance_metric():
+    w = synth.make_workload("tiny", G=1, mode="int", pmin=0, pmax=128, B=700, T=6, dim=64)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 5)
+    ref = H.oracle_outputs(w, 5, tabs, csr)
+    layers = _layers(w, tabs)
+    got = _run(w, layers, csr)
+    _close(layers)
+    _assert_exact(got[0], ref[0])
+    # and the north-star metric against fp64 for a float workload
+    w = synth.make_workload("tiny", G=1, pmin=1, pmax=128, B=300, T=3, dim=32, rows=2000)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 6)
+    layers = _layers(w, tabs)
+    got = _run(w, layers, csr)[0]
+    _close(layers)
+    for t in range(w.T):
+        o, lo, hi = O.rank_table_csr(csr[0][0], t, w.B)
+        z64, S = O.pool_table_f64(tabs[t], o, csr[1][0][lo:hi])
+        assert O.s_normalized_error(got[:, t], z64, S) <= 1e-6
+
+
+def test_identity_routing_and_negative_zero():
+    w = synth.make_workload("tiny", G=1, mode="identity", pmin=1, pmax=1, B=50, T=4)
+    tabs = H.np_tables(w)
+    tabs[2][:] = -0.0  # one-hot of a -0.0 row must return -0.0 bits (C4, P2)
+    csr = H.np_csrs(w, 3)
+    ref = H.oracle_outputs(w, 3, tabs, csr)
+    layers = _layers(w, tabs)
+    got = _run(w, layers, csr)[0]
+    _close(layers)
+    _assert_exact(got, ref[0])
+    assert np.all(np.signbit(got[:, 2]))
+
+
+# ------------------------------------------------------------------------------- simulated G > 1
+@pytest.mark.parametrize("G,flags", [(2, 0), (3, 0), (2, 2), (4, 2)])
+def test_simulated_ranks_bitexact(G, flags):
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=30, B=101, T=7, dim=32, rows=500)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 12)
+    ref = H.oracle_outputs(w, 12, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, csr, flags)
+        for r in range(G):
+            _assert_exact(got[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)
+
+
+def test_placement_invariance_and_rank_without_tables():
+    outs = []
+    for own in ([0, 0, 1, 1, 2, 2], [2, 1, 0, 2, 1, 0], [1, 1, 1, 1, 1, 1], [0, 2, 0, 2, 0, 2]):
+        w = synth.make_workload("tiny", G=3, pmin=0, pmax=20, B=64, T=6, dim=16, owner=np.array(own))
+        tabs = H.np_tables(w)
+        csr = H.np_csrs(w, 44)
+        layers = _layers(w, tabs)
+        got = _run(w, layers, csr)
+        _close(layers)
+        outs.append(np.concatenate(got))
+    for o in outs[1:]:
+        _assert_exact(o, outs[0])
+
+
+def test_epoch_ring_poisoned_slots_exactly_once():
+    """P14: every returned slot is poisoned with NaN after it is read; the 2-slot ring
+    rewrites it two epochs later, so from epoch 2 on every forward lands on poison and
+    must leave no NaN and match the oracle (exactly-once, C21)."""
+    w = synth.make_workload("tiny", G=2, pmin=0, pmax=12, B=90, T=5, dim=32, rows=300)
+    tabs = H.np_tables(w)
+    layers = _layers(w, tabs)
+    try:
+        for epoch in range(6):
+            csr = H.np_csrs(w, 1000 + epoch)
+            ref = H.oracle_outputs(w, 1000 + epoch, tabs, csr)
+            offs, idxs = csr
+            dev_in = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(w.G)]
+            streams = [torch.cuda.Stream() for _ in range(w.G)]
+            torch.cuda.synchronize()
+            ys = [layers[r].forward(dev_in[r][0], dev_in[r][1], 0, streams[r]) for r in range(w.G)]
+            torch.cuda.synchronize()
+            for r in range(w.G):
+                _assert_exact(H.dev_out_to_np(ys[r].clone()), ref[r])
+                ys[r].fill_(float("nan"))
+            torch.cuda.synchronize()
+    finally:
+        _close(layers)
+
+
+def test_bounds_check_flag():
+    w = synth.make_workload("tiny", G=1, pmin=1, pmax=6, B=40, T=2, dim=16, rows=100)
+    tabs = H.np_tables(w)
+    offs, idxs = H.np_csrs(w, 8)
+    bad = idxs[0].copy()
+    bad[3] = 100          # out of range
+    bad[7] = -5
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, ([offs[0]], [bad]), E.EMB_FWD_CHECK_BOUNDS)[0]
+        assert layers[0].device_error(clear=True) & E.EMB_DEVERR_BOUNDS
+        assert layers[0].device_error() == 0
+    finally:
+        _close(layers)
+    # expected: the offending indices contribute nothing
+    for t in range(w.T):
+        o, lo, hi = O.rank_table_csr(offs[0], t, w.B)
+        for b in range(w.B):
+            js = [j for j in range(lo + o[b], lo + o[b + 1]) if 0 <= bad[j] < 100]
+            exp = O.pool_bag_f32(tabs[t][bad[js]]) if js else np.zeros(w.dim, np.float32)
+            assert np.array_equal(np.abs(got[b, t]), np.abs(exp))
+
+
+def test_peer_timeout_sets_error_instead_of_hanging():
+    w = synth.make_workload("tiny", G=2, pmin=1, pmax=4, B=16, T=2, dim=16)
+    tabs = H.np_tables(w)
+    offs, idxs = H.np_csrs(w, 2)
+    layers = _layers(w, tabs, options={"timeout_ms": 200})
+    try:
+        o, x = torch.from_numpy(offs[0]).to(DEV), torch.from_numpy(idxs[0]).to(DEV)
+        layers[0].forward(o, x)        # rank 1 never forwards
+        torch.cuda.synchronize()
+        assert layers[0].device_error(clear=True) & E.EMB_DEVERR_TIMEOUT
+        # rank 1 catches up; both complete epoch 1 (rank 0 then re-runs epoch 2 with rank 1's epoch 2)
+    finally:
+        _close(layers)
+
+
+# ------------------------------------------------------------------------------- comparison path
+def test_baseline_pool_unpack_matches_pgas_bitwise():
+    """P12: pool -> (simulated all-to-all with copies) -> unpack == PGAS output."""
+    G = 3
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=77, T=7, dim=32, rows=400)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 31)
+    ref = H.oracle_outputs(w, 31, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        dev_in = [(torch.from_numpy(csr[0][r]).to(DEV), torch.from_numpy(csr[1][r]).to(DEV)) for r in range(G)]
+        sends, splits = [], []
+        for r in range(G):
+            sc, rc = E.emb_baseline_splits(layers[r].ctx)
+            s = torch.full((max(sum(sc), 1),), float("nan"), device=DEV)
+            E.emb_baseline_pool(layers[r].ctx, dev_in[r][0], dev_in[r][1], s)
+            sends.append(s)
+            splits.append((sc, rc))
+        torch.cuda.synchronize()
+        for r in range(G):  # all_to_all_single semantics, done with copies
+            chunks = []
+            for src in range(G):
+                sc = splits[src][0]
+                off = sum(sc[:r])
+                chunks.append(sends[src][off: off + sc[r]])
+            recv = torch.cat(chunks)
+            assert recv.numel() == sum(splits[r][1])
+            out = torch.full((layers[r].B_r, w.T, w.dim), float("nan"), device=DEV)
+            E.emb_baseline_unpack(layers[r].ctx, recv, out)
+            torch.cuda.synchronize()
+            _assert_exact(out.cpu().numpy(), ref[r])
+    finally:
+        _close(layers)
+
+
+def test_baseline_g1_equals_pgas():
+    w = synth.make_workload("tiny", G=1, pmin=0, pmax=50, B=300, T=4, dim=64, rows=1000, dist="zipf")
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 9)
+    layers = _layers(w, tabs)
+    try:
+        o, x = torch.from_numpy(csr[0][0]).to(DEV), torch.from_numpy(csr[1][0]).to(DEV)
+        a = layers[0].forward(o, x).clone()
+        b = layers[0].forward_baseline(o, x).clone()
+        torch.cuda.synchronize()
+        assert torch.equal(a.view(torch.int32), b.view(torch.int32))
+    finally:
+        _close(layers)
+
+
+def test_forward_host_e2e_matches_device_path():
+    w = synth.make_workload("tiny", G=1, pmin=0, pmax=30, B=500, T=3, dim=64, rows=2000)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 77)
+    ref = H.oracle_outputs(w, 77, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        ho = torch.from_numpy(csr[0][0]).pin_memory()
+        hx = torch.from_numpy(csr[1][0]).pin_memory()
+        hout = torch.empty((w.B, w.T, w.dim), dtype=torch.float32).pin_memory()
+        s = torch.cuda.current_stream()
+        E.emb_forward_host(layers[0].ctx, ho, hx, hout, 0, s)
+        s.synchronize()
+        _assert_exact(hout.numpy(), ref[0])
+    finally:
+        _close(layers)
+
+
+def test_api_errors():
+    with pytest.raises(E.EmbError):
+        E.emb_init(0, 0, 0)
+    ctx = E.emb_init(0, 1, 0)
+    try:
+        with pytest.raises(E.EmbError) as ei:
+            E.emb_forward(ctx, 0, 0)
+        assert ei.value.status == 2  # EMB_ERR_STATE
+        w = torch.zeros((10, 3), device=DEV)
+        with pytest.raises(E.EmbError):
+            E.emb_register_tables(ctx, [10], [0], 3, "f32", "f32", 4, [w])  # 12-byte rows unsupported
+        with pytest.raises(E.EmbError):
+            E.emb_register_tables(ctx, [10], [1], 4, "f32", "f32", 4, [w])  # owner out of range
+        with pytest.raises(E.EmbError):
+            E.emb_set_option(ctx, "nope", 1)
+    finally:
+        E.emb_finalize(ctx)
