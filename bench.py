@@ -1,0 +1,366 @@
+#!/usr/bin/env python
+"""Benchmark of the PGAS-style EMB-layer forward (BASELINE.json metric: EMB fwd
+samples/sec at 1/2/4/8 B200, max over ranks, + % of the HBM/NVLink roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config weak|single|strong|weak_paper|tiny]
+                    [--dist zipf|uniform] [--impl ours|reference]
+    torchrun --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
+
+One JSON line on rank 0.  A "step" is one whole EMB forward (lookup + pool + MP->DP
+exchange, PAPER.md L197 timed scope) over one batch of synthetic Criteo-shaped input
+already resident in HBM; `e2e` repeats it through emb_forward_host with pinned host
+CSR in and the host output out.  `--impl reference` times the CPU oracle (this tier's
+reference arm) on a bounded sample of the same workload.  Nothing here reads
+/root/reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+NVLINK_GBS = 770.0      # measured peer copy per direction (B200_PROFILING.md); nominal 900
+HBM_FALLBACK = 6650.0   # B200_PROFILING.md fallback if MEASURED_PEAKS.json is absent
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=100)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--config", default="weak")
+    p.add_argument("--dist", default=None, help="override index distribution (zipf|uniform)")
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--batches", type=int, default=4, help="distinct pre-generated batches cycled")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-control", action="store_true", help="skip the uniform-index control measurement")
+    p.add_argument("--no-compare", action="store_true", help="skip the NCCL comparison path")
+    p.add_argument("--opt", action="append", default=[], help="libemb option key=value")
+    return p.parse_args()
+
+
+def hbm_peak():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return HBM_FALLBACK, "fallback"
+
+
+def config_desc(w, N):
+    return {"workload": w.name, "tables_total": int(w.T), "tables_per_gpu": int(w.T // max(N, 1)) if w.name != "large" else None,
+            "rows_per_table": int(w.rows[0]), "dim": w.dim, "global_batch": int(w.B), "local_batch": int(w.B // N),
+            "pooling": f"U{{{w.pmin}..{w.pmax}}}", "indices": f"{w.dist}({w.alpha})" if w.dist == "zipf" else "uniform",
+            "weights": w.wdtype, "out": w.odtype, "parallelism": f"table-wise MP x{N} + batch DP x{N}",
+            "aliased": int(w.T // (int(w.phys.max()) + 1)) if int(w.phys.max()) + 1 < w.T else 1,
+            "l2": "inputs larger than L2 (tables >> 126 MB, rotating CSR batches); no flush"}
+
+
+def algorithmic_bytes(w, nnz, nbags, remote_bags):
+    """per lookup d*e + 8 (row + index); per bag 8 (offset) + d*e_o (output)."""
+    e, eo = w.elem_bytes(), w.out_elem_bytes()
+    hbm = nnz * (w.dim * e + 8) + nbags * (8 + w.dim * eo)
+    nvl = remote_bags * w.dim * eo
+    return hbm, nvl
+
+
+# ------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    def __init__(self, device_index: int):
+        self.samples = []
+        self.reasons = set()
+        self._stop = threading.Event()
+        self._th = None
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    _NAMES = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown", 0x4: "sw_power_cap",
+              0x80: "hw_power_brake_slowdown", 0x1: "gpu_idle", 0x2: "applications_clocks_setting"}
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self._NAMES.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.nv:
+            self._th = threading.Thread(target=self._run, daemon=True)
+            self._th.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._th:
+            self._th.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------------ CPU oracle timing
+class OracleSampler:
+    """Time the oracle AS IT STANDS (oracle.emb_oracle, one process, untuned) on k of
+    this rank's tables over the full batch plus the MP->DP layout step; extrapolate
+    to the whole rank workload by table count.  Inputs are generated once, untimed."""
+
+    def __init__(self, w, rank, max_tables=8):
+        from oracle import emb_oracle as O
+        self.O = O
+        self.w = w
+        self.lt = list(w.local_tables(rank))
+        t0 = self.lt[0]
+        self.W = synth.table_rows(w.table_seed, int(w.phys[t0]), int(w.rows[t0]), w.dim, w.mode, w.wdtype)
+        self.csrs = [synth.table_csr(w, w.batch_seed(0), int(t)) for t in self.lt[:max_tables]]
+
+    def run(self, budget_s=12.0, min_tables=1):
+        O, w = self.O, self.w
+        done, Zs, lookups = 0, [], 0
+        t0 = time.perf_counter()
+        while done < len(self.csrs) and (done < min_tables or time.perf_counter() - t0 < budget_s):
+            o, x = self.csrs[done]
+            Zs.append(O.pool_table_f32(self.W, o, x))
+            lookups += int(o[-1])
+            done += 1
+        O.mp_to_dp(Zs, w.G)
+        dt = time.perf_counter() - t0
+        per_rank_s = dt * len(self.lt) / done
+        return {"value": w.B / per_rank_s, "unit": "samples/s", "cores": 1, "kind": "oracle",
+                "sample": f"{done} of {len(self.lt)} local tables x full batch {w.B} ({lookups} lookups; table values "
+                          f"from one physical {int(w.rows[self.lt[0]])}x{w.dim} table) + MP->DP layout, {dt:.2f}s, "
+                          f"extrapolated to the rank's workload by table count",
+                "seconds": dt, "rank_seconds": per_rank_s}
+
+
+def oracle_sample(w, rank, budget_s=12.0):
+    return OracleSampler(w, rank).run(budget_s)
+
+
+def reference_arm(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    N = args.gpus
+    w = synth.make_workload(args.config, G=N, dist=args.dist)
+    smp = OracleSampler(w, 0, max_tables=1)
+    per_step = []
+    cb = None
+    for s in range(args.warmup + args.steps):
+        r = smp.run(budget_s=0.0, min_tables=1)
+        if s >= args.warmup:
+            per_step.append(r["rank_seconds"])
+            cb = r
+    sec = float(np.mean(per_step))
+    val = w.B / sec
+    line = {"impl": "reference", "metric": "EMB fwd samples/sec (max over ranks)", "value": val, "unit": "samples/s",
+            "n_gpus": N, "steps": args.steps, "warmup": args.warmup, "ms_per_step": sec * 1e3,
+            "higher_is_better": True, "scaling": "weak" if args.config.startswith("weak") else "strong",
+            "vs_baseline": None, "dtype": "f32" if w.wdtype == "f32" else "bf16", "data": "synthetic",
+            "config": config_desc(w, N),
+            "cpu_baseline": {"value": val, "unit": "samples/s", "cores": 1, "kind": "oracle",
+                             "sample": "per step: " + cb["sample"]},
+            "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "gpu_launches": 0}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_arm(args)
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_chenbyo24_b200 import emb as E
+    from paper_conf_sc_chenbyo24_b200.comm import torch_allgather
+    from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
+    import synth.gpu as SG
+
+    N = args.gpus
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != N:
+        raise SystemExit(f"--gpus {N} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if N > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    w = synth.make_workload(args.config, G=N, dist=args.dist)
+    stream = torch.cuda.Stream(device=dev)
+
+    # ---- inputs in HBM (untimed)
+    with torch.cuda.stream(stream):
+        tables, _phys = SG.local_tables(w, rank, dev)
+        batches = [SG.rank_csr(w, w.batch_seed(i), rank, dev) for i in range(args.batches)]
+    torch.cuda.synchronize()
+    opts = {}
+    for kv in args.opt:
+        k, v = kv.split("=")
+        opts[k] = int(v)
+    layer = PgasEmbedding(rank, N, local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
+                          torch_allgather() if N > 1 else None, opts)
+    nnz = [int(b[0][-1].item()) for b in batches]
+    T_r = len(w.local_tables(rank))
+    nbags = T_r * w.B
+    B_r = layer.B_r
+    remote_bags = T_r * (w.B - B_r)
+
+    def barrier():
+        if N > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def timed(fn, steps):
+        barrier()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for s in range(steps):
+            fn(s)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        ms = ev0.elapsed_time(ev1) / steps
+        if N > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    def fwd(s):
+        o, x = batches[s % len(batches)]
+        layer.forward(o, x, 0, stream)
+
+    for s in range(args.warmup):
+        fwd(s)
+    barrier()
+    with ClockSampler(local) as clk:
+        ms = timed(fwd, args.steps)
+    assert layer.device_error() == 0, "device error during the timed region"
+    value = w.B / (ms * 1e-3)
+
+    hbm_bytes, nvl_bytes = algorithmic_bytes(w, float(np.mean(nnz)), nbags, remote_bags)
+    peak, peak_kind = hbm_peak()
+    t_hbm = hbm_bytes / (peak * 1e9)
+    t_nvl = nvl_bytes / (NVLINK_GBS * 1e9)
+    bound = "hbm" if t_hbm >= t_nvl else "nvlink"
+    achieved = (hbm_bytes if bound == "hbm" else nvl_bytes) / (ms * 1e-3) / 1e9
+    pk = peak if bound == "hbm" else NVLINK_GBS
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            tj = json.load(f)
+        key = f"{w.name}:{w.dist}:G{N}"
+        if key in tj:
+            traffic = tj[key]["dram_bytes_per_launch"]
+    except Exception:
+        pass
+    roof = {"bound": bound, "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": achieved / pk,
+            "traffic": traffic, "kernel": "emb_fwd_kernel (fused gather+pool+store+flags)",
+            "algorithmic_bytes_per_launch": hbm_bytes if bound == "hbm" else nvl_bytes,
+            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else "measured peer copy 770 GB/s (B200_PROFILING.md)",
+            "t_roof_ms": max(t_hbm, t_nvl) * 1e3, "frac_of_roofline_time": max(t_hbm, t_nvl) * 1e3 / ms}
+
+    extra = {}
+    # ---- uniform-index control (lookup bytes ~= DRAM bytes; no zipf reuse)
+    if not args.no_control and w.dist == "zipf":
+        wu = synth.make_workload(args.config, G=N, dist="uniform")
+        with torch.cuda.stream(stream):
+            ub = [SG.rank_csr(wu, wu.batch_seed(100 + i), rank, dev) for i in range(2)]
+        torch.cuda.synchronize()
+        for s in range(3):
+            layer.forward(ub[s % 2][0], ub[s % 2][1], 0, stream)
+
+        def fwd_u(s):
+            layer.forward(ub[s % 2][0], ub[s % 2][1], 0, stream)
+        ms_u = timed(fwd_u, max(args.steps // 2, 3))
+        hb_u, _ = algorithmic_bytes(wu, float(np.mean([int(b[0][-1].item()) for b in ub])), nbags, remote_bags)
+        extra["uniform_control"] = {"ms_per_step": ms_u, "value": w.B / (ms_u * 1e-3),
+                                    "achieved_gbs": hb_u / (ms_u * 1e-3) / 1e9, "frac": hb_u / (ms_u * 1e-3) / 1e9 / peak}
+        del ub
+
+    # ---- conventional comparison path: pool kernel -> NCCL all_to_all_single -> unpack kernel
+    if not args.no_compare:
+        def fwd_b(s):
+            o, x = batches[s % len(batches)]
+            with torch.cuda.stream(stream):
+                layer.forward_baseline(o, x, None, 0, stream)
+        for s in range(3):
+            fwd_b(s)
+        ms_b = timed(fwd_b, max(args.steps // 2, 3))
+        extra["comparison_nccl_path"] = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3),
+                                         "pgas_speedup": ms_b / ms,
+                                         "note": "G=1: pool kernel only (no exchange, no unpack)" if N == 1 else
+                                         "pool kernel + NCCL all_to_all_single + unpack kernel"}
+
+    # ---- e2e through the public C ABI with host buffers
+    e2e = None
+    if not args.no_e2e:
+        hb = []
+        for o, x in batches[:2]:
+            hb.append((o.cpu().pin_memory(), x.cpu().pin_memory()))
+        hout = torch.empty((B_r, w.T, w.dim), dtype=layer.out_dtype).pin_memory()
+
+        def fwd_h(s):
+            ho, hx = hb[s % 2]
+            E.emb_forward_host(layer.ctx, ho, hx, hout, 0, stream)
+        for s in range(2):
+            fwd_h(s)
+        k_e2e = max(min(args.steps, 20), 3)
+        ms_e = timed(fwd_h, k_e2e)
+        h2d = float(np.mean([(ho.numel() + hx.numel()) * 8 for ho, hx in hb]))
+        d2h = B_r * w.T * w.dim * w.out_elem_bytes()
+        e2e = {"value": w.B / (ms_e * 1e-3), "unit": "samples/s", "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": ms_e, "steps": k_e2e,
+               "path": "emb_forward_host: pinned H2D of offsets+indices, fused kernel, D2H of Y_r, one stream"}
+
+    cpu = None
+    if rank == 0 and N == 1 and not args.no_cpu_baseline:
+        cpu = oracle_sample(w, 0)
+
+    layer.close()
+    if N > 1:
+        dist.barrier()
+    if rank == 0:
+        line = {"metric": "EMB fwd samples/sec (max over ranks)", "value": value, "unit": "samples/s", "n_gpus": N,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None,
+                "dtype": "f32" if (w.wdtype == "f32") else "bf16", "data": "synthetic",
+                "config": config_desc(w, N), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": args.steps, "clocks": clk.summary(), **extra}
+        print(json.dumps(line), flush=True)
+    if N > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

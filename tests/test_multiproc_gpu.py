@@ -1,0 +1,89 @@
+"""Real cross-process PGAS on ONE GPU: G rank processes bound to cuda:0 exchange CUDA
+IPC handles over a gloo process group, and the fused kernel's "remote" stores and
+release/acquire flags go through cudaIpcOpenMemHandle mappings of the other
+processes' symmetric buffers (SURVEY §4 'multi-rank without a cluster')."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, G, port, q, flags, owner, epochs):
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    try:
+        import torch.distributed as dist
+
+        import emb_test_helpers as H
+        import synth
+        from paper_conf_sc_chenbyo24_b200 import emb as E
+        from paper_conf_sc_chenbyo24_b200.comm import torch_allgather
+        from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
+
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=G)
+        w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=97, T=6, dim=32, rows=600,
+                                owner=np.array(owner) if owner else None)
+        tabs = H.np_tables(w)
+        dev = torch.device("cuda", 0)
+        local = [torch.from_numpy(tabs[int(w.phys[t])]).to(dev) for t in w.local_tables(rank)]
+        layer = PgasEmbedding(rank, G, 0, w.rows, w.owner, w.dim, local, w.B, "f32", "f32", torch_allgather(),
+                              {"timeout_ms": 20000})
+        ok = True
+        s = torch.cuda.Stream()
+        for ep in range(epochs):
+            o, x = synth.rank_csr(w, 500 + ep, rank)
+            ref = H.oracle_outputs(w, 500 + ep, tabs)[rank]
+            y = layer.forward(torch.from_numpy(o).to(dev), torch.from_numpy(x).to(dev), flags, s)
+            if flags & E.EMB_FWD_SEPARATE_WAIT:
+                layer.wait(s)
+            s.synchronize()
+            got = y.cpu().numpy()
+            ok = ok and np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+            y.fill_(float("nan"))
+            torch.cuda.synchronize()
+            dist.barrier()  # consumer of slot e&1 done before anyone runs e+2 (stream order across processes)
+        err = layer.device_error()
+        layer.close()
+        dist.destroy_process_group()
+        q.put((rank, bool(ok), int(err), ""))
+    except Exception as e:  # report instead of hanging the parent
+        import traceback
+        q.put((rank, False, -1, traceback.format_exc()))
+
+
+@pytest.mark.parametrize("G,flags,owner", [(2, 0, None), (3, 0, [2, 2, 0, 1, 0, 2]), (2, 2, None)])
+def test_cross_process_ipc_pgas(G, flags, owner):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_worker, args=(r, G, port, q, flags, owner, 4)) for r in range(G)]
+    for p in ps:
+        p.start()
+    res = []
+    for _ in range(G):
+        res.append(q.get(timeout=240))
+    for p in ps:
+        p.join(timeout=60)
+    for rank, ok, err, tb in sorted(res):
+        assert tb == "", tb
+        assert ok, f"rank {rank} output != oracle"
+        assert err == 0, f"rank {rank} device error {err}"
