@@ -152,7 +152,11 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
 /* Tunables (take effect on the next launch): "chunk_rows" (target rows per claimed
  * work chunk, default 256), "ctas_per_sm" (0 = occupancy max), "stagger" (1 =
  * destination-staggered chunk order, default), "timeout_ms" (peer wait, default
- * 10000 or env EMB_TIMEOUT_MS), "unroll" (rows in flight per warp: 4, 8 or 16). */
+ * 10000 or env EMB_TIMEOUT_MS), "unroll" (row pipeline: 0 = auto (default), 2 or 4 = rows per group of the
+ * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
+ * flight per warp in a cp.async shared-memory ring), "minblocks" (CTAs of 256 per
+ * SM the register budget is sized for: 0 = auto (4 for one vector per lane, else 1), 1, 4, 6).
+ * Errors: EMB_ERR_ARG for an unknown key or value. */
 emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
 
 /* Read (after synchronizing the forward's stream) and optionally clear the sticky

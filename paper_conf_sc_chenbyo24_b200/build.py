@@ -18,9 +18,12 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC", "-ftz=false", "-prec-div=true",
          "-prec-sqrt=true", "-fmad=false", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
 
+CSRC = os.path.join(PKG, "csrc")
 LIBS = {
-    "emb": dict(srcs=[os.path.join(PKG, "csrc", "emb_runtime.cu")],
-                deps=[os.path.join(PKG, "csrc", "emb_kernels.cuh"), os.path.join(ROOT, "include", "emb.h")],
+    "emb": dict(srcs=[os.path.join(CSRC, f) for f in ("emb_runtime.cu", "emb_inst_f32_f32.cu", "emb_inst_f32_bf16.cu",
+                                                       "emb_inst_bf16_f32.cu", "emb_inst_bf16_bf16.cu")],
+                deps=[os.path.join(CSRC, "emb_kernels.cuh"), os.path.join(CSRC, "emb_dispatch.h"),
+                      os.path.join(ROOT, "include", "emb.h")],
                 out=os.path.join(PKG, "libemb.so")),
     "synth": dict(srcs=[os.path.join(ROOT, "synth", "csrc", "synth_gen.cu")],
                   deps=[os.path.join(ROOT, "include", "synth.h")],
@@ -36,23 +39,38 @@ def _stale(spec) -> bool:
     return any(os.path.getmtime(s) > t for s in spec["srcs"] + spec["deps"] if os.path.exists(s))
 
 
+def _nvcc(args):
+    r = subprocess.run([NVCC, *args], capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("nvcc failed: " + " ".join(args[-3:]))
+    return r.stderr
+
+
 def build(names=None, force: bool = False, verbose: bool = False) -> None:
+    """Compile every translation unit to an object in parallel, then link the .so."""
+    from concurrent.futures import ThreadPoolExecutor
     for name, spec in LIBS.items():
         if names and name not in names:
             continue
         if not force and not _stale(spec):
             continue
-        cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), *spec["srcs"], "-o", spec["out"] + ".tmp"]
-        r = subprocess.run(cmd, capture_output=True, text=True)
-        if r.returncode != 0:
-            sys.stderr.write(r.stdout + r.stderr)
-            raise RuntimeError(f"nvcc failed for {name}")
+        objdir = os.path.join(os.path.dirname(spec["out"]), ".obj")
+        os.makedirs(objdir, exist_ok=True)
+        comp = [f for f in FLAGS if f != "-shared"]
+        jobs = []
+        for src in spec["srcs"]:
+            obj = os.path.join(objdir, os.path.basename(src) + ".o")
+            jobs.append((obj, [*ARCH, *comp, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]))
+        with ThreadPoolExecutor(max_workers=min(len(jobs), os.cpu_count() or 4)) as ex:
+            logs = list(ex.map(lambda j: _nvcc(j[1]), jobs))
+        _nvcc([*ARCH, "-shared", "-Xcompiler", "-fPIC", *[j[0] for j in jobs], "-o", spec["out"] + ".tmp"])
         os.replace(spec["out"] + ".tmp", spec["out"])
         log = os.path.join(os.path.dirname(spec["out"]), f".{name}_ptxas.log")
         with open(log, "w") as f:
-            f.write(r.stderr)
+            f.write("".join(logs))
         if verbose:
-            sys.stdout.write(r.stderr)
+            sys.stdout.write("".join(logs))
 
 
 if __name__ == "__main__":

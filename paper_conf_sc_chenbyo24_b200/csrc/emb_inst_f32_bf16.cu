@@ -1,0 +1,41 @@
+// emb_inst_f32_bf16.cu -- instantiations of the fused kernel for f32 tables, bf16 output.
+#include "emb_dispatch.h"
+
+namespace emb {
+namespace {
+template <int VB, int NV, typename WT, typename OT, bool CHECK>
+KernelFn pick_u(int unroll, int mb, bool full) {
+  if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 4, false>;  // rows narrower than a warp
+  if (unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, CHECK, 6, true>;
+  switch (mb) {
+    case 1: return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 1, true>;
+    case 6: return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 6, true>;
+    default: return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 4, true>;
+  }
+}
+template <int VB, int NV, typename WT, typename OT>
+KernelFn pick_c(int unroll, bool check, int mb, bool full) {
+  if (unroll >= 8) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
+    if constexpr (NV == 1) {
+      if (unroll == 16)
+        return check ? emb_fwd_async_kernel<VB, NV, WT, OT, 16, true, 3> : emb_fwd_async_kernel<VB, NV, WT, OT, 16, false, 3>;
+      return check ? emb_fwd_async_kernel<VB, NV, WT, OT, 8, true, 4> : emb_fwd_async_kernel<VB, NV, WT, OT, 8, false, 4>;
+    }
+    unroll = 4;
+  }
+  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full) : pick_u<VB, NV, WT, OT, false>(unroll, mb, full);
+}
+}  // namespace
+
+KernelFn pick_tile_f32_bf16(int vb, int nv, int unroll, bool check, int mb, bool full) {
+  using WT = float;
+  using OT = __nv_bfloat16;
+  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full);
+  switch (nv) {
+    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full);
+    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full);
+    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full);
+    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full);
+  }
+}
+}  // namespace emb

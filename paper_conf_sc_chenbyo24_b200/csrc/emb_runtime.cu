@@ -11,6 +11,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -19,7 +20,9 @@
 #include <vector>
 
 #include "../../include/emb.h"
+#define EMB_RUNTIME_TU
 #include "emb_kernels.cuh"
+#include "emb_dispatch.h"
 
 using namespace emb;
 
@@ -78,7 +81,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 8;
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -109,40 +112,26 @@ struct emb_ctx {
   } while (0)
 
 static size_t esize(emb_dtype_t t) { return t == EMB_F32 ? 4 : 2; }
+// register budget per tile: one vector per lane fits 64 registers (4 CTAs of 256 per SM,
+// no spills for any dtype pair); wider rows keep the unconstrained build
+static int eff_minblocks(const emb_ctx* c) { return c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1); }
+// rows per pipeline group: 4 rows for both 8- and 16-byte lane vectors (measured best)
+static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4); }
+// a row exactly covers the warp's 32 lane vectors (lets the row stride be a constant)
+static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
+// shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
+static size_t dyn_smem(const emb_ctx* c) {
+  return (eff_unroll(c) >= 8 && c->nv == 1) ? (size_t)(kBlock / 32) * c->unroll * 32 * c->vb : 0;
+}
 
 // ---------------------------------------------------------------------------- kernel dispatch
 namespace {
 
-using KernelFn = void (*)(FwdParams);
-
-template <int VB, int NV, typename WT, typename OT>
-KernelFn pick_u(int unroll, bool check) {
-  switch (unroll) {
-    case 4:
-      return check ? emb_fwd_kernel<VB, NV, WT, OT, 4, true> : emb_fwd_kernel<VB, NV, WT, OT, 4, false>;
-    case 16:
-      return check ? emb_fwd_kernel<VB, NV, WT, OT, 16, true> : emb_fwd_kernel<VB, NV, WT, OT, 16, false>;
-    default:
-      return check ? emb_fwd_kernel<VB, NV, WT, OT, 8, true> : emb_fwd_kernel<VB, NV, WT, OT, 8, false>;
-  }
-}
-
-template <typename WT, typename OT>
-KernelFn pick_tile(int vb, int nv, int unroll, bool check) {
-  if (vb == 8) return pick_u<8, 1, WT, OT>(unroll, check);
-  switch (nv) {
-    case 2: return pick_u<16, 2, WT, OT>(unroll, check);
-    case 4: return pick_u<16, 4, WT, OT>(unroll, check);
-    case 8: return pick_u<16, 8, WT, OT>(unroll, check);
-    default: return pick_u<16, 1, WT, OT>(unroll, check);
-  }
-}
-
-KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check) {
-  if (w == EMB_F32 && o == EMB_F32) return pick_tile<float, float>(vb, nv, unroll, check);
-  if (w == EMB_F32 && o == EMB_BF16) return pick_tile<float, __nv_bfloat16>(vb, nv, unroll, check);
-  if (w == EMB_BF16 && o == EMB_F32) return pick_tile<__nv_bfloat16, float>(vb, nv, unroll, check);
-  return pick_tile<__nv_bfloat16, __nv_bfloat16>(vb, nv, unroll, check);
+KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full) {
+  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full);
+  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full);
+  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full);
+  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full);
 }
 
 // row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
@@ -381,14 +370,16 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 }
 
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, c->unroll, (flags & EMB_FWD_CHECK_BOUNDS) != 0);
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c));
+  const size_t smem = dyn_smem(c);
+  if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0) {
-    CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0));
+    CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem));
     if (per_sm < 1) per_sm = 1;
   }
   const int grid = c->num_sms * per_sm;
-  k<<<grid, kBlock, 0, s>>>(p);
+  k<<<grid, kBlock, smem, s>>>(p);
   CK(c, cudaGetLastError());
   return EMB_OK;
 }
@@ -504,8 +495,10 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   i->epoch = c->epoch;
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0 && c->registered) {
-    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, c->unroll, false);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0);
+    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c));
+    const size_t smem = dyn_smem(c);
+    if (smem > 0) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem);
   }
   i->grid = c->num_sms * std::max(per_sm, 1);
   i->block = kBlock;
@@ -521,7 +514,14 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "ctas_per_sm")) { if (v < 0 || v > 32) FAIL(c, EMB_ERR_ARG, "ctas_per_sm"); c->ctas_per_sm = (int)v; }
   else if (!strcmp(key, "stagger")) c->stagger = v ? 1 : 0;
   else if (!strcmp(key, "timeout_ms")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "timeout_ms < 1"); c->timeout_ns = v * 1000000ll; }
-  else if (!strcmp(key, "unroll")) { if (v != 4 && v != 8 && v != 16) FAIL(c, EMB_ERR_ARG, "unroll must be 4, 8 or 16"); c->unroll = (int)v; }
+  else if (!strcmp(key, "unroll")) {
+    if (v != 0 && v != 2 && v != 4 && v != 8 && v != 16) FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline) or 8, 16 (shared-memory ring)");
+    c->unroll = (int)v;
+  }
+  else if (!strcmp(key, "minblocks")) {
+    if (v != 0 && v != 1 && v != 4 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4 or 6");
+    c->minblocks = (int)v;
+  }
   else FAIL(c, EMB_ERR_ARG, "unknown option '%s'", key);
   return EMB_OK;
 }

@@ -325,3 +325,31 @@ def test_api_errors():
             E.emb_set_option(ctx, "nope", 1)
     finally:
         E.emb_finalize(ctx)
+
+
+VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),
+                 dict(dim=64, pmin=1, pmax=40, B=257, rows=2000),
+                 dict(dim=128, wdtype="bf16", odtype="bf16", pmin=0, pmax=50, B=129, rows=1000),
+                 dict(dim=32, pmin=0, pmax=9, B=100)]
+
+
+@pytest.mark.parametrize("opts", [{"unroll": 2}, {"unroll": 4}, {"unroll": 8}, {"unroll": 16},
+                                  {"unroll": 4, "minblocks": 1}, {"unroll": 4, "minblocks": 6},
+                                  {"chunk_rows": 1}, {"chunk_rows": 100000}, {"stagger": 0}])
+@pytest.mark.parametrize("case", range(len(VARIANT_CASES)))
+def test_pipeline_variants_bitexact(opts, case):
+    """Every register/shared-memory pipeline variant and chunking is bit-exact."""
+    w = synth.make_workload("tiny", G=2, T=5, **VARIANT_CASES[case])
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 71)
+    ref = H.oracle_outputs(w, 71, tabs, csr)
+    layers = _layers(w, tabs, options=opts)
+    try:
+        got = _run(w, layers, csr)
+        got_chk = _run(w, layers, csr, E.EMB_FWD_CHECK_BOUNDS)
+        for r in range(w.G):
+            _assert_exact(got[r], ref[r])
+            _assert_exact(got_chk[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)
