@@ -121,7 +121,7 @@ static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb 
 static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
 static size_t dyn_smem(const emb_ctx* c) {
-  return (eff_unroll(c) >= 8 && c->nv == 1) ? (size_t)(kBlock / 32) * c->unroll * 32 * c->vb : 0;
+  return (eff_unroll(c) >= 8 && c->nv == 1) ? (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb : 0;
 }
 
 // ---------------------------------------------------------------------------- kernel dispatch
