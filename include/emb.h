@@ -141,6 +141,19 @@ emb_status_t emb_wait(emb_ctx_t* ctx, void* stream);
 emb_status_t emb_forward_host(emb_ctx_t* ctx, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
                               void* stream, void* h_out);
 
+/* Pipelined end-to-end path (same inputs/outputs as emb_forward_host): call k's H2D
+ * (internal copy-in stream, two alternating device stages) overlaps call k-1's kernel
+ * (on `stream`) and call k-2's D2H (internal copy-out stream).  h_out of a call is
+ * complete once emb_host_drain(ctx, s) has been called and `s` synchronized (or after a
+ * later call's drain).  The host input buffers of a call must stay unchanged, and its
+ * h_out must not be reused by another in-flight call, until then; h_out buffers should
+ * be pinned.  Two calls in flight at most per stage (the library waits on events). */
+emb_status_t emb_forward_host_async(emb_ctx_t* ctx, const int64_t* h_offsets, const int64_t* h_indices,
+                                    uint32_t flags, void* stream, void* h_out);
+
+/* Make `stream` wait for every outstanding copy of emb_forward_host_async. */
+emb_status_t emb_host_drain(emb_ctx_t* ctx, void* stream);
+
 /* Collective: waits for the device, unmaps peers, frees everything, destroys ctx. */
 emb_status_t emb_finalize(emb_ctx_t* ctx);
 

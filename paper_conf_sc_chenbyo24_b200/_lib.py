@@ -40,6 +40,8 @@ SIGNATURES = {
     "emb_forward": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(C.c_void_p)]),
     "emb_wait": (C.c_int, [C.c_void_p, C.c_void_p]),
     "emb_forward_host": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
+    "emb_forward_host_async": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
+    "emb_host_drain": (C.c_int, [C.c_void_p, C.c_void_p]),
     "emb_finalize": (C.c_int, [C.c_void_p]),
     "emb_local_batch": (C.c_int, [C.c_void_p, C.c_int, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
     "emb_get_info": (C.c_int, [C.c_void_p, C.POINTER(EmbInfo)]),

@@ -92,6 +92,14 @@ struct emb_ctx {
   int64_t* d_off_stage = nullptr;
   int64_t* d_idx_stage = nullptr;
   size_t idx_cap = 0;
+  // pipelined host path: two input stages, copy-in / copy-out streams, events
+  int64_t* p_off[2] = {nullptr, nullptr};
+  int64_t* p_idx[2] = {nullptr, nullptr};
+  size_t p_cap[2] = {0, 0};
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
+  bool kern_rec[2] = {false, false}, out_rec[2] = {false, false};
+  uint64_t host_calls = 0;
   std::string err;
   FwdParams last{};
 };
@@ -442,6 +450,75 @@ emb_status_t emb_forward_host(emb_ctx_t* c, const int64_t* h_offsets, const int6
   return EMB_OK;
 }
 
+emb_status_t emb_forward_host_async(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
+                                    void* stream, void* h_out) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward_host_async before emb_register_tables");
+  if (!h_offsets || !h_out || (c->T_r > 0 && !h_indices)) FAIL(c, EMB_ERR_ARG, "NULL host buffer");
+  CK(c, cudaSetDevice(c->dev));
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!c->s_in) {
+    CK(c, cudaStreamCreateWithFlags(&c->s_in, cudaStreamNonBlocking));
+    CK(c, cudaStreamCreateWithFlags(&c->s_out, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CK(c, cudaEventCreateWithFlags(&c->ev_in[i], cudaEventDisableTiming));
+      CK(c, cudaEventCreateWithFlags(&c->ev_kern[i], cudaEventDisableTiming));
+      CK(c, cudaEventCreateWithFlags(&c->ev_out[i], cudaEventDisableTiming));
+    }
+  }
+  const int k = (int)(c->host_calls & 1);
+  const size_t noff = (size_t)c->T_r * (size_t)c->B + 1;
+  const int64_t nnz = h_offsets[noff - 1];
+  if (nnz < 0) FAIL(c, EMB_ERR_ARG, "negative nnz");
+  if (!c->p_off[k] || (size_t)nnz > c->p_cap[k]) {  // (re)allocate stage k: drain everything first
+    CK(c, cudaStreamSynchronize(c->s_in));
+    CK(c, cudaStreamSynchronize(c->s_out));
+    CK(c, cudaStreamSynchronize(s));
+    if (!c->p_off[k]) CK(c, cudaMalloc(&c->p_off[k], noff * sizeof(int64_t)));
+    if (c->p_idx[k]) CK(c, cudaFree(c->p_idx[k]));
+    c->p_cap[k] = std::max<size_t>((size_t)nnz, 1) + (size_t)nnz / 4;
+    CK(c, cudaMalloc(&c->p_idx[k], c->p_cap[k] * sizeof(int64_t)));
+  }
+  // 1. H2D into stage k once the kernel that last read it (two calls ago) is done
+  if (c->kern_rec[k]) CK(c, cudaStreamWaitEvent(c->s_in, c->ev_kern[k], 0));
+  CK(c, cudaMemcpyAsync(c->p_off[k], h_offsets, noff * sizeof(int64_t), cudaMemcpyHostToDevice, c->s_in));
+  if (nnz > 0)
+    CK(c, cudaMemcpyAsync(c->p_idx[k], h_indices, (size_t)nnz * sizeof(int64_t), cudaMemcpyHostToDevice, c->s_in));
+  CK(c, cudaEventRecord(c->ev_in[k], c->s_in));
+  // 2. forward on the caller's stream after the inputs landed and after the D2H that last
+  //    read this epoch's output slot (2-slot ring) finished
+  const int slot = (int)((c->epoch + 1) & 1);
+  CK(c, cudaStreamWaitEvent(s, c->ev_in[k], 0));
+  if (c->out_rec[slot]) CK(c, cudaStreamWaitEvent(s, c->ev_out[slot], 0));
+  void* dout = nullptr;
+  emb_status_t st = emb_forward(c, c->p_off[k], c->p_idx[k], flags, stream, &dout);
+  if (st != EMB_OK) return st;
+  if (flags & EMB_FWD_SEPARATE_WAIT) {
+    st = emb_wait(c, stream);
+    if (st != EMB_OK) return st;
+  }
+  CK(c, cudaEventRecord(c->ev_kern[k], s));
+  c->kern_rec[k] = true;
+  // 3. D2H of Y_r on the copy-out stream, overlapping the next call's H2D and kernel
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  CK(c, cudaStreamWaitEvent(c->s_out, c->ev_kern[k], 0));
+  CK(c, cudaMemcpyAsync(h_out, dout, (size_t)Br * c->T * c->d * esize(c->odt), cudaMemcpyDeviceToHost, c->s_out));
+  CK(c, cudaEventRecord(c->ev_out[slot], c->s_out));
+  c->out_rec[slot] = true;
+  c->host_calls += 1;
+  return EMB_OK;
+}
+
+emb_status_t emb_host_drain(emb_ctx_t* c, void* stream) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->s_in) return EMB_OK;
+  CK(c, cudaSetDevice(c->dev));
+  cudaStream_t s = (cudaStream_t)stream;
+  for (int i = 0; i < 2; ++i)
+    if (c->out_rec[i]) CK(c, cudaStreamWaitEvent(s, c->ev_out[i], 0));
+  return EMB_OK;
+}
+
 emb_status_t emb_finalize(emb_ctx_t* c) {
   if (!c) return EMB_ERR_ARG;
   cudaSetDevice(c->dev);
@@ -461,6 +538,15 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->d_unpack_stride) cudaFree(c->d_unpack_stride);
   if (c->d_off_stage) cudaFree(c->d_off_stage);
   if (c->d_idx_stage) cudaFree(c->d_idx_stage);
+  for (int i = 0; i < 2; ++i) {
+    if (c->p_off[i]) cudaFree(c->p_off[i]);
+    if (c->p_idx[i]) cudaFree(c->p_idx[i]);
+    if (c->ev_in[i]) cudaEventDestroy(c->ev_in[i]);
+    if (c->ev_kern[i]) cudaEventDestroy(c->ev_kern[i]);
+    if (c->ev_out[i]) cudaEventDestroy(c->ev_out[i]);
+  }
+  if (c->s_in) cudaStreamDestroy(c->s_in);
+  if (c->s_out) cudaStreamDestroy(c->s_out);
   delete c;
   return st;
 }

@@ -129,6 +129,17 @@ def emb_forward_host(ctx: EmbCtx, h_offsets, h_indices, h_out, flags: int = 0, s
     _check(ctx, st)
 
 
+def emb_forward_host_async(ctx: EmbCtx, h_offsets, h_indices, h_out, flags: int = 0, stream=None) -> None:
+    """Pipelined host path: H2D / kernel / D2H of consecutive calls overlap."""
+    st = _lib.lib().emb_forward_host_async(ctx, _ptr(h_offsets), _ptr(h_indices), int(flags), _stream(stream),
+                                           _ptr(h_out))
+    _check(ctx, st)
+
+
+def emb_host_drain(ctx: EmbCtx, stream=None) -> None:
+    _check(ctx, _lib.lib().emb_host_drain(ctx, _stream(stream)))
+
+
 def emb_finalize(ctx: EmbCtx) -> None:
     if ctx.ptr:
         st = _lib.lib().emb_finalize(ctx)

@@ -353,3 +353,24 @@ def test_pipeline_variants_bitexact(opts, case):
             assert layers[r].device_error() == 0
     finally:
         _close(layers)
+
+
+def test_forward_host_async_pipeline_matches_oracle():
+    """Pipelined host path: 5 calls in flight on alternating stages, each its own h_out."""
+    w = synth.make_workload("tiny", G=1, pmin=0, pmax=30, B=300, T=3, dim=64, rows=2000)
+    tabs = H.np_tables(w)
+    layers = _layers(w, tabs)
+    try:
+        seeds = [900 + i for i in range(5)]
+        csrs = [H.np_csrs(w, sd) for sd in seeds]
+        hin = [(torch.from_numpy(c[0][0]).pin_memory(), torch.from_numpy(c[1][0]).pin_memory()) for c in csrs]
+        houts = [torch.full((w.B, w.T, w.dim), float("nan")).pin_memory() for _ in seeds]
+        s = torch.cuda.current_stream()
+        for i in range(len(seeds)):
+            E.emb_forward_host_async(layers[0].ctx, hin[i][0], hin[i][1], houts[i], 0, s)
+        E.emb_host_drain(layers[0].ctx, s)
+        s.synchronize()
+        for i, sd in enumerate(seeds):
+            _assert_exact(houts[i].numpy(), H.oracle_outputs(w, sd, tabs, csrs[i])[0])
+    finally:
+        _close(layers)
