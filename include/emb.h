@@ -169,8 +169,15 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
  * flight per warp in a cp.async shared-memory ring), "minblocks" (CTAs of 256 per
  * SM the register budget is sized for: 0 = auto (4 for one vector per lane, else 1), 1, 4, 6).
+ * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
+ * of that many records and makes every warp append {globaltimer ns, bytes stored to
+ * peers << 32 | bytes stored locally} after each claimed chunk; 0 disables).
  * Errors: EMB_ERR_ARG for an unknown key or value. */
 emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
+
+/* f1: synchronize the device, copy up to `capacity` trace records (2 x uint64 each,
+ * see "trace_capacity") into `host`, set *count, and reset the trace. */
+emb_status_t emb_trace_read(emb_ctx_t* ctx, uint64_t* host, int64_t capacity, int64_t* count);
 
 /* Read (after synchronizing the forward's stream) and optionally clear the sticky
  * device error word (EMB_DEVERR_* bits). */

@@ -100,6 +100,9 @@ struct emb_ctx {
   cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
   bool kern_rec[2] = {false, false}, out_rec[2] = {false, false};
   uint64_t host_calls = 0;
+  // f1 trace buffer
+  unsigned long long* trace = nullptr;
+  uint32_t trace_cap = 0;
   std::string err;
   FwdParams last{};
 };
@@ -374,6 +377,8 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
       p->out_base[g] = send + (size_t)c->bstart[g] * (size_t)c->T_r * (size_t)c->d * osz;
   }
   p->epoch = (uint32_t)c->epoch;
+  p->trace = c->trace;
+  p->trace_cap = c->trace_cap;
   return EMB_OK;
 }
 
@@ -519,6 +524,20 @@ emb_status_t emb_host_drain(emb_ctx_t* c, void* stream) {
   return EMB_OK;
 }
 
+emb_status_t emb_trace_read(emb_ctx_t* c, uint64_t* host, int64_t capacity, int64_t* count) {
+  if (!c || !count || (capacity > 0 && !host)) return EMB_ERR_ARG;
+  CK(c, cudaSetDevice(c->dev));
+  CK(c, cudaDeviceSynchronize());
+  unsigned n = 0;
+  CK(c, cudaMemcpy(&n, &c->ctrl->trace_n, sizeof(unsigned), cudaMemcpyDeviceToHost));
+  const int64_t have = std::min<int64_t>((int64_t)n, (int64_t)c->trace_cap);
+  const int64_t m = std::min<int64_t>(have, capacity);
+  if (m > 0) CK(c, cudaMemcpy(host, c->trace, (size_t)m * 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  *count = m;
+  CK(c, cudaMemset(&c->ctrl->trace_n, 0, sizeof(unsigned)));
+  return EMB_OK;
+}
+
 emb_status_t emb_finalize(emb_ctx_t* c) {
   if (!c) return EMB_ERR_ARG;
   cudaSetDevice(c->dev);
@@ -546,6 +565,7 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
     if (c->ev_out[i]) cudaEventDestroy(c->ev_out[i]);
   }
   if (c->s_in) cudaStreamDestroy(c->s_in);
+  if (c->trace) cudaFree(c->trace);
   if (c->s_out) cudaStreamDestroy(c->s_out);
   delete c;
   return st;
@@ -607,6 +627,19 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "minblocks")) {
     if (v != 0 && v != 1 && v != 4 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4 or 6");
     c->minblocks = (int)v;
+  }
+  else if (!strcmp(key, "trace_capacity")) {
+    if (v < 0 || v > (1 << 26)) FAIL(c, EMB_ERR_ARG, "trace_capacity in [0, 2^26]");
+    CK(c, cudaSetDevice(c->dev));
+    CK(c, cudaDeviceSynchronize());
+    if (c->trace) CK(c, cudaFree(c->trace));
+    c->trace = nullptr;
+    c->trace_cap = 0;
+    if (v > 0) {
+      CK(c, cudaMalloc(&c->trace, (size_t)v * 2 * sizeof(unsigned long long)));
+      c->trace_cap = (uint32_t)v;
+    }
+    CK(c, cudaMemset(&c->ctrl->trace_n, 0, sizeof(unsigned)));
   }
   else FAIL(c, EMB_ERR_ARG, "unknown option '%s'", key);
   return EMB_OK;

@@ -170,6 +170,15 @@ def emb_query_device_error(ctx: EmbCtx, clear: bool = False) -> int:
     return w.value
 
 
+def emb_trace_read(ctx: EmbCtx, capacity: int):
+    """f1 trace: numpy uint64 [n, 2] = {globaltimer ns, remote_bytes << 32 | local_bytes}."""
+    import numpy as np
+    buf = np.zeros((max(int(capacity), 1), 2), dtype=np.uint64)
+    n = C.c_int64()
+    _check(ctx, _lib.lib().emb_trace_read(ctx, buf.ctypes.data, int(capacity), C.byref(n)))
+    return buf[: n.value]
+
+
 def emb_last_error(ctx: Optional[EmbCtx]) -> str:
     return (_lib.lib().emb_last_error(ctx.ptr if ctx is not None else None) or b"").decode(errors="replace")
 

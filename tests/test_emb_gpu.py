@@ -374,3 +374,32 @@ def test_forward_host_async_pipeline_matches_oracle():
             _assert_exact(houts[i].numpy(), H.oracle_outputs(w, sd, tabs, csrs[i])[0])
     finally:
         _close(layers)
+
+
+def test_trace_counts_every_stored_byte():
+    """f1: per-chunk trace records add up to exactly the bytes each rank stores, split into
+    local and remote by destination, with monotone globaltimer stamps inside the forward."""
+    G = 2
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=20, B=200, T=6, dim=32, rows=500)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 5)
+    layers = _layers(w, tabs, options={"trace_capacity": 100000})
+    try:
+        got = _run(w, layers, csr)
+        ref = H.oracle_outputs(w, 5, tabs, csr)
+        for r in range(G):
+            _assert_exact(got[r], ref[r])
+            tr = E.emb_trace_read(layers[r].ctx, 100000)
+            assert tr.shape[0] > 0
+            remote = int((tr[:, 1] >> np.uint64(32)).sum())
+            local = int((tr[:, 1] & np.uint64(0xFFFFFFFF)).sum())
+            Tr = len(w.local_tables(r))
+            starts, counts = O.split_batch(w.B, G)
+            vec = w.dim * 4
+            assert local == Tr * counts[r] * vec
+            assert remote == Tr * (w.B - counts[r]) * vec
+            assert np.all(tr[:, 0] > 0)
+        # reading resets the trace
+        assert E.emb_trace_read(layers[0].ctx, 10).shape[0] == 0
+    finally:
+        _close(layers)
