@@ -57,10 +57,19 @@ def main():
             for i in range(a.steps):
                 fn(i)
             e1.record(s)
+            try:
+                import pynvml
+                pynvml.nvmlInit()
+                h = pynvml.nvmlDeviceGetHandleByIndex(0)
+                clk = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000
+            except Exception:
+                clk = pw = None
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / a.steps
             print(json.dumps({"config": a.config, "dist": dist, "opts": o, "ms": round(ms, 4),
-                              "Msamples_s": round(w.B / ms / 1e3, 3), "GBs": round(byt / ms / 1e6, 1)}), flush=True)
+                              "Msamples_s": round(w.B / ms / 1e3, 3), "GBs": round(byt / ms / 1e6, 1),
+                              "sm_mhz": clk, "power_w": pw}), flush=True)
             assert layer.device_error() == 0
     layer.close()
 
