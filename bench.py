@@ -47,6 +47,10 @@ def parse():
     p.add_argument("--no-control", action="store_true", help="skip the uniform-index control measurement")
     p.add_argument("--no-compare", action="store_true", help="skip the NCCL comparison path")
     p.add_argument("--opt", action="append", default=[], help="libemb option key=value")
+    p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                   help="process-group backend (gloo: test harness only; a2a staged through host)")
+    p.add_argument("--same-device", action="store_true",
+                   help="test harness: every rank on cuda:0 (N>1 on a 1-GPU box; ranks time-slice)")
     return p.parse_args()
 
 
@@ -231,10 +235,15 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != N:
         raise SystemExit(f"--gpus {N} but WORLD_SIZE={world}")
+    if args.same_device:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if N > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     w = synth.make_workload(args.config, G=N, dist=args.dist)
     stream = torch.cuda.Stream(device=dev)
 
@@ -273,7 +282,7 @@ def main():
         torch.cuda.synchronize()
         ms = ev0.elapsed_time(ev1) / steps
         if N > 1:
-            t = torch.tensor([ms], device=dev)
+            t = torch.tensor([ms], device=dev if args.backend == "nccl" else "cpu")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
         return ms
@@ -354,7 +363,9 @@ def main():
         extra["comparison_nccl_path"] = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3),
                                          "pgas_speedup": ms_b / ms,
                                          "note": "G=1: pool kernel only (no exchange, no unpack)" if N == 1 else
-                                         "pool kernel + NCCL all_to_all_single + unpack kernel"}
+                                         f"pool kernel + {args.backend} all_to_all_single + unpack kernel"
+                                         + (" (gloo: host-staged test harness, not a measurement)"
+                                            if args.backend == "gloo" else "")}
 
     # ---- e2e through the public C ABI with host buffers
     e2e = None

@@ -78,9 +78,16 @@ class PgasEmbedding:
         if self.ctx.world_size == 1:  # G = 1: send already is [B][T][d]; no exchange, no unpack
             return send[: self.B_r * self.T * self.dim].view(self.B_r, self.T, self.dim)
         import torch.distributed as dist
-        work = dist.all_to_all_single(recv, send, output_split_sizes=self._recv_counts,
-                                      input_split_sizes=self._send_counts, group=group, async_op=True)
-        work.wait()
+        if dist.get_backend(group) == "nccl":
+            work = dist.all_to_all_single(recv, send, output_split_sizes=self._recv_counts,
+                                          input_split_sizes=self._send_counts, group=group, async_op=True)
+            work.wait()
+        else:  # gloo (CPU test harness): stage the exchange through host memory
+            torch.cuda.current_stream(self.device).synchronize() if stream is None else stream.synchronize()
+            hs, hr = send.cpu(), torch.empty(recv.shape, dtype=recv.dtype)
+            dist.all_to_all_single(hr, hs, output_split_sizes=self._recv_counts,
+                                   input_split_sizes=self._send_counts, group=group)
+            recv.copy_(hr)
         E.emb_baseline_unpack(self.ctx, recv, out, stream)
         return out
 
