@@ -169,11 +169,41 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
  * flight per warp in a cp.async shared-memory ring), "minblocks" (CTAs of 256 per
  * SM the register budget is sized for: 0 = auto (4 for one vector per lane, else 1), 1, 4, 6).
+ * "enable_backward" (f2: 1 before emb_register_tables adds two fp32 grad slots
+ * [B_r][T][d] to the symmetric buffer for emb_backward),
  * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
  * of that many records and makes every warp append {globaltimer ns, bytes stored to
  * peers << 32 | bytes stored locally} after each claimed chunk; 0 disables).
  * Errors: EMB_ERR_ARG for an unknown key or value. */
 emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
+
+/* ---- f2: backward (§V) ---------------------------------------------
+ * dW_t[x, :] += sum over bags (t, b) and positions j with x_t[j] = x of dY[b, t, :].
+ * Usage per step (collective, every rank in the same order):
+ *   emb_backward_grad_slot(ctx, stream, &dY)  -> device fp32 [B_r][T][d] slot of THIS
+ *       rank's gradient w.r.t. its outputs; write it with work on `stream` (the call
+ *       enqueues a wait until every peer finished reading the slot's previous use);
+ *   emb_backward_grad_ready(ctx, stream) -> releases "my dY is written" to every peer
+ *       (stream-ordered after the fill);
+ *   emb_backward(ctx, offsets, indices, dW, flags, stream) -> one fused kernel acquires
+ *       every peer's "ready" flag and, per local bag, loads the
+ *       bag's gradient vector from the DP rank's slot (one-sided NVLink load) and
+ *       atomically adds it (red.add.f32, FTZ per the hardware atomic) into the rows of
+ *       dW[t_l] (caller-owned device fp32 [M_t][d], NOT zeroed by the library; 16-byte
+ *       aligned) for every index of the bag.  Same CSR as emb_forward.  Accumulation
+ *       order is unspecified (atomics): results match the oracle within the fp32
+ *       tolerance, exactly for integer-valued gradients.
+ * Every CTA of the fused kernel waits for the peers' "ready" flags before it starts, so
+ * when several ranks share ONE GPU (test harnesses) all ranks' grad_ready calls must be
+ * issued before any rank's emb_backward.  The last CTA releases "done reading" into each
+ * peer (emb_backward_grad_slot waits on it before a slot is refilled).
+ * Requires "enable_backward" before emb_register_tables.  Errors: EMB_ERR_STATE (also for
+ * emb_backward without a preceding grad_ready), EMB_ERR_ARG, EMB_ERR_CUDA; peer timeouts
+ * set EMB_DEVERR_TIMEOUT. */
+emb_status_t emb_backward_grad_slot(emb_ctx_t* ctx, void* stream, void** dY);
+emb_status_t emb_backward_grad_ready(emb_ctx_t* ctx, void* stream);
+emb_status_t emb_backward(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, void* const* dW,
+                          uint32_t flags, void* stream);
 
 /* f1: synchronize the device, copy up to `capacity` trace records (2 x uint64 each,
  * see "trace_capacity") into `host`, set *count, and reset the trace. */

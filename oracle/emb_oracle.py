@@ -32,7 +32,10 @@ closed forms (P2-P4), integer tables exact in any order (P5), identity routing (
 power-of-two scaling (P7), linearity (P8), placement invariance (P9), rank concat
 (P10), torch.nn.functional.embedding_bag + gloo all_to_all special cases (P11),
 conservation (P13), the paper's Fig. 3 / Fig. 4 structure (P15), and torch's bf16
-conversion for the rounding step.
+conversion for the rounding step.  Backward (§V):
+`emb_backward` is the transpose of the pooling + layout conversion, pinned by a
+pure-Python loop, the adjoint identity <pool(W), dY> = <W, dW> (exact on integer data),
+torch autograd of embedding_bag(mode="sum"), and placement invariance.
 """
 from __future__ import annotations
 
@@ -43,7 +46,7 @@ import numpy as np
 __all__ = [
     "validate_csr", "pool_table_f32", "pool_table_f64", "rne_bf16", "bf16_to_f32",
     "split_batch", "rank_table_csr", "mp_to_dp", "emb_forward", "pool_bag_f32",
-    "pool_bag_f64", "s_normalized_error",
+    "pool_bag_f64", "s_normalized_error", "emb_backward",
 ]
 
 
@@ -202,3 +205,38 @@ def s_normalized_error(y: np.ndarray, y_ref: np.ndarray, S: np.ndarray) -> float
     with np.errstate(divide="ignore", invalid="ignore"):
         q = np.where(diff == 0, 0.0, diff / S)
     return float(np.max(q)) if q.size else 0.0
+
+
+# ----------------------------------------------------------------------------- backward (f2)
+def emb_backward(rows: Sequence[int], dim: int, owner: Sequence[int], rank_offsets: Sequence[np.ndarray],
+                 rank_indices: Sequence[np.ndarray], dY: Sequence[np.ndarray], B: int, G: int):
+    """Adjoint of the forward (§V L378-382 for the exchange; the arithmetic is the
+    transpose of sum pooling, L91-95):
+
+        dW_t[x, :] = sum_{b} sum_{j in bag(t, b), x_t[j] = x} dY[b, t, :]
+
+    dY[r] is rank r's gradient w.r.t. its outputs, [B_r][T][d] (data parallel, C8 split);
+    the bags come from the owner's CSR (C11).  Returns (dW64, S, count): per global table
+    the fp64 gradient [M_t][d], S = sum |dY| per element (tolerance denominator) and the
+    number of contributions per row (for the order-independent error bound n*2^-24*S)."""
+    T = len(rows)
+    owner = [int(o) for o in owner]
+    dY_full = np.concatenate([np.asarray(y, dtype=np.float64) for y in dY], axis=0)   # [B][T][d]
+    assert dY_full.shape == (B, T, dim)
+    dW, S, cnt = [], [], []
+    for t in range(T):
+        dW.append(np.zeros((int(rows[t]), dim)))
+        S.append(np.zeros((int(rows[t]), dim)))
+        cnt.append(np.zeros(int(rows[t]), dtype=np.int64))
+    for r in range(G):
+        local = [t for t in range(T) if owner[t] == r]
+        for tl, t in enumerate(local):
+            o, lo, hi = rank_table_csr(rank_offsets[r], tl, B)
+            x = np.asarray(rank_indices[r][lo:hi], dtype=np.int64)
+            validate_csr(o, x, int(rows[t]))
+            bag_of = np.repeat(np.arange(B), np.diff(o))          # sample of every position
+            g = dY_full[bag_of, t, :]
+            np.add.at(dW[t], x, g)
+            np.add.at(S[t], x, np.abs(g))
+            np.add.at(cnt[t], x, 1)
+    return dW, S, cnt

@@ -48,6 +48,9 @@ SIGNATURES = {
     "emb_set_option": (C.c_int, [C.c_void_p, C.c_char_p, C.c_int64]),
     "emb_query_device_error": (C.c_int, [C.c_void_p, C.POINTER(C.c_uint32), C.c_int]),
     "emb_last_error": (C.c_char_p, [C.c_void_p]),
+    "emb_backward_grad_slot": (C.c_int, [C.c_void_p, C.c_void_p, C.POINTER(C.c_void_p)]),
+    "emb_backward_grad_ready": (C.c_int, [C.c_void_p, C.c_void_p]),
+    "emb_backward": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.POINTER(C.c_void_p), C.c_uint32, C.c_void_p]),
     "emb_trace_read": (C.c_int, [C.c_void_p, C.c_void_p, C.c_int64, C.POINTER(C.c_int64)]),
     "emb_baseline_splits": (C.c_int, [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
     "emb_baseline_pool": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),

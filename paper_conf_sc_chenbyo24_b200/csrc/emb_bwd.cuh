@@ -1,0 +1,189 @@
+// emb_bwd.cuh -- SURVEY row f2: the EMB-layer backward with PGAS-style one-sided access.
+//
+// PAPER.md §V (L378-382): "during backpropagation, the gradients for these embeddings need
+// to be communicated back to the GPUs that own these embeddings ... gradients must be
+// aggregated ... replacing multiple rounds of collective calls with atomic PGAS
+// direct-GPU remote [accesses]".  Definition (adjoint of sum pooling, L91-95):
+//     dW_t[x, :] = sum over bags (t, b), positions j with x_t[j] = x, of dY[b, t, :]
+// where dY[b] lives on the rank owning sample b (data parallel) and dW_t on the owner of
+// table t (model parallel).
+//
+// B200 design: the OWNER pulls.  Every rank writes its dY [B_r][T][d] (fp32) into a
+// symmetric grad slot and releases a per-source "ready" flag; the owner's fused kernel
+// acquires the flags, then per bag loads the bag's gradient vector straight from the DP
+// rank's slot (one-sided NVLink load; the load of the next bag is in flight while the
+// current one is scattered) and red.add.v4.f32's it into the dW rows of every index of
+// the bag (L2 atomics, no sort, no all-to-all, no unpack).  The last CTA releases a
+// per-source "done" flag so each DP rank knows when its slot may be refilled.
+#pragma once
+
+#include "emb_kernels.cuh"
+
+namespace emb {
+
+struct BwdParams {
+  const TableDesc* tables;     // [T_r] (rows, global id)
+  float* const* dW;            // [T_r] device pointers, fp32 [M_t][d], accumulated into
+  const int64_t* offsets;      // [T_r*B + 1]
+  const int64_t* indices;
+  int64_t B;
+  int64_t bstart[kMaxG + 1];
+  const char* gsrc[kMaxG];     // per DP rank: its grad slot of this epoch, [B_dst][T][d] fp32
+  uint32_t* peer_ready[kMaxG]; // &ready_p[rank] on peer p
+  uint32_t* peer_done[kMaxG];  // &done_p[rank] on peer p
+  const uint32_t* my_ready;    // ready_r[G]
+  Ctrl* ctrl;                  // uses bwork / bdone
+  int64_t timeout_ns;
+  int32_t T, T_r, d, G, rank, lanes, chunk_rows;
+  uint32_t epoch;
+};
+
+template <int VB>
+__device__ __forceinline__ void red_add_vec(float* p, const uint32_t* r);
+template <>
+__device__ __forceinline__ void red_add_vec<16>(float* p, const uint32_t* r) {
+  asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(__uint_as_float(r[0])),
+               "f"(__uint_as_float(r[1])), "f"(__uint_as_float(r[2])), "f"(__uint_as_float(r[3]))
+               : "memory");
+}
+template <>
+__device__ __forceinline__ void red_add_vec<8>(float* p, const uint32_t* r) {
+  asm volatile("red.relaxed.gpu.global.add.v2.f32 [%0], {%1,%2};" ::"l"(p), "f"(__uint_as_float(r[0])),
+               "f"(__uint_as_float(r[1]))
+               : "memory");
+}
+template <int VB>
+__device__ __forceinline__ void ld_vec_relaxed(const void* p, uint32_t* r);
+template <>
+__device__ __forceinline__ void ld_vec_relaxed<16>(const void* p, uint32_t* r) {
+  asm volatile("ld.global.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_vec_relaxed<8>(const void* p, uint32_t* r) {
+  asm volatile("ld.global.v2.b32 {%0,%1}, [%2];" : "=r"(r[0]), "=r"(r[1]) : "l"(p));
+}
+
+__device__ __forceinline__ bool wait_flags_geq(const uint32_t* flags, int G, int rank, uint32_t epoch, int64_t timeout_ns,
+                                               unsigned* err) {
+  const uint64_t t0 = globaltimer();
+  for (int s = 0; s < G; ++s) {
+    if (s == rank) continue;
+    unsigned ns = 32;
+    while ((int32_t)(ld_relaxed_sys(flags + s) - epoch) < 0) {
+      if ((int64_t)(globaltimer() - t0) > timeout_ns) {
+        atomicOr(err, 0x1u);
+        return false;
+      }
+      __nanosleep(ns);
+      if (ns < 1024) ns <<= 1;
+    }
+  }
+  fence_acq_rel_sys();
+  return true;
+}
+
+// VB bytes per lane vector, NV vectors per lane (row = 32*VB*NV bytes when all lanes active)
+template <int VB, int NV>
+__global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__ BwdParams p) {
+  constexpr int W = VB / 4;
+  const int lane = threadIdx.x & 31;
+  const bool active = lane < p.lanes;
+  const int64_t rowbytes = (int64_t)p.d * 4;
+  const int64_t B = p.B;
+  // acquire every DP rank's dY of this epoch
+  if (threadIdx.x == 0 && p.G > 1) wait_flags_geq(p.my_ready, p.G, p.rank, p.epoch, p.timeout_ns, &p.ctrl->err);
+  __syncthreads();
+
+  const int64_t nbags = (int64_t)p.T_r * B;
+  if (nbags > 0) {
+    const int64_t nnz = __ldg(p.offsets + nbags);
+    const int64_t cb64 = (nnz > 0) ? ((int64_t)p.chunk_rows * nbags + nnz - 1) / nnz : 31;
+    const int cb = (int)(cb64 < 1 ? 1 : (cb64 > 31 ? 31 : cb64));
+    const int64_t cpt = (B + cb - 1) / cb;
+    const int64_t nchunks = cpt * p.T_r;
+    for (;;) {
+      unsigned c = 0;
+      if (lane == 0) c = atomicAdd(&p.ctrl->bwork, 1u);
+      c = __shfl_sync(kFull, c, 0);
+      if ((int64_t)c >= nchunks) break;
+      const int t_l = (int)(c / cpt);
+      const int64_t b0 = ((int64_t)c % cpt) * cb;
+      const int nb = (int)min((int64_t)cb, B - b0);
+      const int64_t o_l = (lane <= nb) ? ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane) : 0;
+      const TableDesc* tdp = p.tables + t_l;
+      const int64_t tglob = __ldg(&tdp->tglob);
+      char* dwl = reinterpret_cast<char*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t_l))) + lane * VB;
+
+      auto gaddr = [&](int bag) -> const char* {        // dY[b][tglob] on the DP rank owning b
+        const int64_t b = b0 + bag;
+        int dst = 0;
+        while (b >= p.bstart[dst + 1]) ++dst;
+        return p.gsrc[dst] + ((b - p.bstart[dst]) * p.T + tglob) * rowbytes + lane * VB;
+      };
+      uint32_t gn[NV][W];
+      if (active) {
+        const char* a = gaddr(0);
+#pragma unroll
+        for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
+      }
+      const int64_t pos0 = __shfl_sync(kFull, o_l, 0);
+      int64_t pos = pos0;
+      int64_t batch = -1;                                 // first position held in `my`
+      uint32_t my = 0;
+      for (int bag = 0; bag < nb; ++bag) {
+        uint32_t g[NV][W];
+#pragma unroll
+        for (int v = 0; v < NV; ++v)
+#pragma unroll
+          for (int i = 0; i < W; ++i) g[v][i] = gn[v][i];
+        if (bag + 1 < nb && active) {                     // next bag's gradient in flight
+          const char* a = gaddr(bag + 1);
+#pragma unroll
+          for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
+        }
+        const int64_t end = __shfl_sync(kFull, o_l, bag + 1);
+        for (; pos < end; ++pos) {
+          if (pos >= batch + 32 || batch < 0) {
+            batch = pos;
+            my = (pos + lane < __shfl_sync(kFull, o_l, nb)) ? (uint32_t)ld_stream_i64(p.indices + pos + lane) : 0u;
+          }
+          const uint32_t x = __shfl_sync(kFull, my, (int)(pos - batch));
+          if (active) {
+            char* rp = dwl + (uint64_t)x * (uint64_t)rowbytes;
+#pragma unroll
+            for (int v = 0; v < NV; ++v) red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), g[v]);
+          }
+        }
+      }
+    }
+  }
+  // completion: every CTA's reads of peer slots are done before the last CTA tells the
+  // peers their slots may be refilled
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  fence_acq_rel_sys();
+  const unsigned prev = atomicAdd(&p.ctrl->bdone, 1u);
+  if (prev != gridDim.x - 1) return;
+  fence_acq_rel_sys();
+  p.ctrl->bdone = 0;
+  p.ctrl->bwork = 0;
+  for (int q = 1; q < p.G; ++q) st_release_sys(p.peer_done[(p.rank + q) % p.G], p.epoch);
+}
+
+#ifdef EMB_RUNTIME_TU
+// release "my dY of this epoch is in my grad slot" to every peer (stream-ordered after the
+// kernels that wrote it)
+__global__ void emb_bwd_signal_kernel(const __grid_constant__ BwdParams p) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  fence_acq_rel_sys();
+  for (int q = 1; q < p.G; ++q) st_release_sys(p.peer_ready[(p.rank + q) % p.G], p.epoch);
+}
+// before a grad slot is refilled: wait until every peer finished reading its previous use
+__global__ void emb_bwd_slot_wait_kernel(const uint32_t* my_done, int G, int rank, uint32_t epoch, int64_t timeout_ns,
+                                         unsigned* err) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  wait_flags_geq(my_done, G, rank, epoch, timeout_ns, err);
+}
+#endif
+
+}  // namespace emb

@@ -23,6 +23,7 @@
 #define EMB_RUNTIME_TU
 #include "emb_kernels.cuh"
 #include "emb_dispatch.h"
+#include "emb_bwd.cuh"
 
 using namespace emb;
 
@@ -38,6 +39,8 @@ struct PeerBlob {
   uint64_t bytes;
   uint64_t slot_off;     // byte offset of slot 0
   uint64_t slot_bytes;   // bytes per slot (B_r*T*d*e_o rounded up to 256)
+  uint64_t grad_off;     // byte offset of backward grad slot 0 (0 = backward not enabled)
+  uint64_t gslot_bytes;  // bytes per grad slot (B_r*T*d*4 rounded up)
   int32_t device;
   int32_t pad;
   cudaIpcMemHandle_t handle;
@@ -100,6 +103,15 @@ struct emb_ctx {
   cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
   bool kern_rec[2] = {false, false}, out_rec[2] = {false, false};
   uint64_t host_calls = 0;
+  // f2 backward
+  bool bwd_enabled = false;
+  size_t grad_off = 0, gslot_bytes = 0;
+  std::vector<uint64_t> peer_grad_off, peer_gslot_bytes;
+  uint64_t bepoch = 0;
+  bool bwd_ready_pending = false;
+  float** d_dW = nullptr;
+  std::vector<void*> h_dW;
+  int blanes = 32, bvb = 16, bnv = 1;
   // f1 trace buffer
   unsigned long long* trace = nullptr;
   uint32_t trace_cap = 0;
@@ -276,9 +288,17 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   }
   // symmetric buffer: [flags: G u32, padded to 512 B][slot 0][slot 1]
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  // header: [fwd flags G u32 @0][bwd ready G u32 @64][bwd done G u32 @128], 512 B
   c->slot_off = 512;
   c->slot_bytes = round_up((size_t)Br * (size_t)num_tables * (size_t)dim * osz, 512);
   c->sym_bytes = c->slot_off + 2 * c->slot_bytes;
+  if (c->bwd_enabled) {
+    if (!choose_tiling((int64_t)dim * 4, 4, 4, &c->blanes, &c->bvb, &c->bnv) || c->bnv > 4)
+      FAIL(c, EMB_ERR_ARG, "backward: unsupported fp32 row size %d bytes", dim * 4);
+    c->grad_off = c->sym_bytes;
+    c->gslot_bytes = round_up((size_t)Br * (size_t)num_tables * (size_t)dim * 4, 512);
+    c->sym_bytes += 2 * c->gslot_bytes;
+  }
   {
     cudaError_t e = cudaMalloc(&c->sym, c->sym_bytes);
     if (e == cudaErrorMemoryAllocation) FAIL(c, EMB_ERR_NOMEM, "symmetric buffer of %zu bytes: out of memory", c->sym_bytes);
@@ -295,6 +315,8 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   mine.bytes = c->sym_bytes;
   mine.slot_off = c->slot_off;
   mine.slot_bytes = c->slot_bytes;
+  mine.grad_off = c->grad_off;
+  mine.gslot_bytes = c->gslot_bytes;
   mine.device = c->dev;
   CK(c, cudaIpcGetMemHandle(&mine.handle, c->sym));
   std::vector<PeerBlob> all(c->G);
@@ -307,12 +329,17 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   c->peer_slot_off.assign(c->G, 0);
   c->peer_slot_bytes.assign(c->G, 0);
   c->peer_ipc.assign(c->G, false);
+  c->peer_grad_off.assign(c->G, 0);
+  c->peer_gslot_bytes.assign(c->G, 0);
   for (int p = 0; p < c->G; ++p) {
     const PeerBlob& b = all[p];
     if (b.magic != kMagic || b.rank != p) FAIL(c, EMB_ERR_PEER, "bad peer blob from rank %d", p);
     if (b.host_hash != mine.host_hash) FAIL(c, EMB_ERR_PEER, "rank %d is on another host (multi-node is out of scope)", p);
     c->peer_slot_off[p] = b.slot_off;
     c->peer_slot_bytes[p] = b.slot_bytes;
+    c->peer_grad_off[p] = b.grad_off;
+    c->peer_gslot_bytes[p] = b.gslot_bytes;
+    if ((b.grad_off != 0) != c->bwd_enabled) FAIL(c, EMB_ERR_PEER, "rank %d disagrees on enable_backward", p);
     if (p == c->rank) {
       c->peer_base[p] = c->sym;
     } else if (b.pid == mine.pid) {  // simulated rank in this process: raw pointer
@@ -524,6 +551,100 @@ emb_status_t emb_host_drain(emb_ctx_t* c, void* stream) {
   return EMB_OK;
 }
 
+static void fill_bwd_params(emb_ctx_t* c, BwdParams* p) {
+  memset(p, 0, sizeof(*p));
+  p->tables = c->d_tables;
+  p->dW = c->d_dW;
+  p->B = c->B;
+  for (int g = 0; g <= c->G; ++g) p->bstart[g] = c->bstart[g];
+  for (int g = c->G + 1; g <= kMaxG; ++g) p->bstart[g] = INT64_MAX;
+  const int slot = (int)(c->bepoch & 1);
+  for (int g = 0; g < c->G; ++g) {
+    p->gsrc[g] = c->peer_base[g] + c->peer_grad_off[g] + (size_t)slot * c->peer_gslot_bytes[g];
+    p->peer_ready[g] = (g == c->rank) ? nullptr : reinterpret_cast<uint32_t*>(c->peer_base[g] + 64) + c->rank;
+    p->peer_done[g] = (g == c->rank) ? nullptr : reinterpret_cast<uint32_t*>(c->peer_base[g] + 128) + c->rank;
+  }
+  p->my_ready = reinterpret_cast<const uint32_t*>(c->sym + 64);
+  p->ctrl = c->ctrl;
+  p->timeout_ns = c->timeout_ns;
+  p->T = c->T;
+  p->T_r = c->T_r;
+  p->d = c->d;
+  p->G = c->G;
+  p->rank = c->rank;
+  p->lanes = c->blanes;
+  p->chunk_rows = c->chunk_rows;
+  p->epoch = (uint32_t)c->bepoch;
+}
+
+emb_status_t emb_backward_grad_slot(emb_ctx_t* c, void* stream, void** dY) {
+  if (!c || !dY) return EMB_ERR_ARG;
+  if (!c->registered || !c->bwd_enabled) FAIL(c, EMB_ERR_STATE, "backward not enabled (set enable_backward before registering)");
+  CK(c, cudaSetDevice(c->dev));
+  const uint64_t next = c->bepoch + 1;
+  // the slot of epoch `next` was last read by the peers at epoch next-2
+  if (c->G > 1 && next > 2) {
+    emb_bwd_slot_wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(reinterpret_cast<const uint32_t*>(c->sym + 128), c->G,
+                                                                  c->rank, (uint32_t)(next - 2), c->timeout_ns,
+                                                                  &c->ctrl->err);
+    CK(c, cudaGetLastError());
+  }
+  *dY = c->sym + c->grad_off + (size_t)(next & 1) * c->gslot_bytes;
+  return EMB_OK;
+}
+
+emb_status_t emb_backward_grad_ready(emb_ctx_t* c, void* stream) {
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered || !c->bwd_enabled) FAIL(c, EMB_ERR_STATE, "backward not enabled (set enable_backward before registering)");
+  if (c->bwd_ready_pending) FAIL(c, EMB_ERR_STATE, "emb_backward_grad_ready called twice without emb_backward");
+  CK(c, cudaSetDevice(c->dev));
+  c->bepoch += 1;
+  c->bwd_ready_pending = true;
+  if (c->G > 1) {
+    BwdParams p;
+    fill_bwd_params(c, &p);
+    emb_bwd_signal_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(p);
+    CK(c, cudaGetLastError());
+  }
+  return EMB_OK;
+}
+
+emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, void* const* dW,
+                          uint32_t flags, void* stream) {
+  (void)flags;
+  if (!c) return EMB_ERR_ARG;
+  if (!c->registered || !c->bwd_enabled) FAIL(c, EMB_ERR_STATE, "backward not enabled (set enable_backward before registering)");
+  if (!c->bwd_ready_pending) FAIL(c, EMB_ERR_STATE, "emb_backward without emb_backward_grad_ready");
+  if (c->T_r > 0 && (!offsets || !indices || !dW)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
+  CK(c, cudaSetDevice(c->dev));
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!c->d_dW) CK(c, cudaMalloc(&c->d_dW, std::max(c->T_r, 1) * sizeof(float*)));
+  bool same = (int)c->h_dW.size() == c->T_r;
+  for (int i = 0; same && i < c->T_r; ++i) same = c->h_dW[i] == dW[i];
+  if (!same) {
+    for (int i = 0; i < c->T_r; ++i)
+      if (!dW[i] || ((uintptr_t)dW[i]) % 16) FAIL(c, EMB_ERR_ARG, "dW[%d] NULL or not 16-byte aligned", i);
+    c->h_dW.assign(dW, dW + c->T_r);
+    CK(c, cudaStreamSynchronize(s));
+    CK(c, cudaMemcpy(c->d_dW, c->h_dW.data(), c->T_r * sizeof(float*), cudaMemcpyHostToDevice));
+  }
+  c->bwd_ready_pending = false;
+  BwdParams p;
+  fill_bwd_params(c, &p);
+  p.offsets = offsets;
+  p.indices = indices;
+  void (*k)(BwdParams) = nullptr;
+  if (c->bvb == 8) k = emb_bwd_kernel<8, 1>;
+  else if (c->bnv == 2) k = emb_bwd_kernel<16, 2>;
+  else if (c->bnv == 4) k = emb_bwd_kernel<16, 4>;
+  else k = emb_bwd_kernel<16, 1>;
+  int per_sm = 0;
+  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0));
+  k<<<c->num_sms * std::max(per_sm, 1), kBlock, 0, s>>>(p);
+  CK(c, cudaGetLastError());
+  return EMB_OK;
+}
+
 emb_status_t emb_trace_read(emb_ctx_t* c, uint64_t* host, int64_t capacity, int64_t* count) {
   if (!c || !count || (capacity > 0 && !host)) return EMB_ERR_ARG;
   CK(c, cudaSetDevice(c->dev));
@@ -566,6 +687,7 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   }
   if (c->s_in) cudaStreamDestroy(c->s_in);
   if (c->trace) cudaFree(c->trace);
+  if (c->d_dW) cudaFree(c->d_dW);
   if (c->s_out) cudaStreamDestroy(c->s_out);
   delete c;
   return st;
@@ -627,6 +749,10 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "minblocks")) {
     if (v != 0 && v != 1 && v != 4 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4 or 6");
     c->minblocks = (int)v;
+  }
+  else if (!strcmp(key, "enable_backward")) {
+    if (c->registered) FAIL(c, EMB_ERR_STATE, "enable_backward must be set before emb_register_tables");
+    c->bwd_enabled = v != 0;
   }
   else if (!strcmp(key, "trace_capacity")) {
     if (v < 0 || v > (1 << 26)) FAIL(c, EMB_ERR_ARG, "trace_capacity in [0, 2^26]");

@@ -170,6 +170,23 @@ def emb_query_device_error(ctx: EmbCtx, clear: bool = False) -> int:
     return w.value
 
 
+def emb_backward_grad_slot(ctx: EmbCtx, stream=None) -> int:
+    """Device address of this rank's fp32 [B_r][T][d] gradient slot for the next backward."""
+    out = C.c_void_p()
+    _check(ctx, _lib.lib().emb_backward_grad_slot(ctx, _stream(stream), C.byref(out)))
+    return out.value
+
+
+def emb_backward_grad_ready(ctx: EmbCtx, stream=None) -> None:
+    _check(ctx, _lib.lib().emb_backward_grad_ready(ctx, _stream(stream)))
+
+
+def emb_backward(ctx: EmbCtx, offsets, indices, dW: Sequence, flags: int = 0, stream=None) -> None:
+    n = len(dW)
+    arr = (C.c_void_p * max(n, 1))(*[_ptr(x) for x in dW])
+    _check(ctx, _lib.lib().emb_backward(ctx, _ptr(offsets), _ptr(indices), arr, int(flags), _stream(stream)))
+
+
 def emb_trace_read(ctx: EmbCtx, capacity: int):
     """f1 trace: numpy uint64 [n, 2] = {globaltimer ns, remote_bytes << 32 | local_bytes}."""
     import numpy as np

@@ -37,9 +37,11 @@ class PgasEmbedding:
 
     def __init__(self, rank: int, world_size: int, device: int, rows: Sequence[int], owner: Sequence[int], dim: int,
                  local_weights: Sequence[torch.Tensor], global_batch: int, weight_dtype="f32", out_dtype="f32",
-                 allgather=None, options: Optional[dict] = None):
+                 allgather=None, options: Optional[dict] = None, backward: bool = False):
         self.device = torch.device("cuda", device)
         self.ctx = E.emb_init(rank, world_size, device, allgather)
+        if backward:
+            E.emb_set_option(self.ctx, "enable_backward", 1)
         self._weights = list(local_weights)  # zero-copy: keep alive
         E.emb_register_tables(self.ctx, rows, owner, dim, weight_dtype, out_dtype, global_batch, self._weights)
         for k, v in (options or {}).items():
@@ -90,6 +92,26 @@ class PgasEmbedding:
             recv.copy_(hr)
         E.emb_baseline_unpack(self.ctx, recv, out, stream)
         return out
+
+    # ---- f2 backward (§V) ---------------------------------------------
+    def grad_slot(self, stream=None) -> torch.Tensor:
+        """fp32 [B_r][T][d] view of this rank's output-gradient slot for the next backward;
+        fill it on `stream` before calling backward()."""
+        ptr = E.emb_backward_grad_slot(self.ctx, stream)
+        return wrap_device(ptr, (self.B_r, self.T, self.dim), torch.float32, self.device)
+
+    def grad_ready(self, stream=None) -> None:
+        """Publish this rank's filled gradient slot to the peers (release)."""
+        E.emb_backward_grad_ready(self.ctx, stream)
+
+    def backward(self, offsets: torch.Tensor, indices: torch.Tensor, dW: Sequence[torch.Tensor], flags: int = 0,
+                 stream=None, publish: bool = True) -> None:
+        """Accumulate dL/dW of this rank's tables into dW[t_l] (fp32 [M_t][d]).  With
+        publish=True the slot is published first (one rank per GPU); ranks sharing a GPU
+        call grad_ready() on all ranks first and pass publish=False."""
+        if publish:
+            E.emb_backward_grad_ready(self.ctx, stream)
+        E.emb_backward(self.ctx, offsets, indices, list(dW), flags, stream)
 
     def device_error(self, clear: bool = False) -> int:
         return E.emb_query_device_error(self.ctx, clear)

@@ -337,3 +337,72 @@ def test_validate_rejects_bad_csr():
 def test_split_batch_rule():
     assert O.split_batch(10, 3) == ([0, 4, 7], [4, 3, 3])
     assert O.split_batch(16384 * 8, 8)[1] == [16384] * 8
+
+
+# ------------------------------------------------------------------------------- backward (f2)
+def _dY(w, seed, integer=True):
+    rng = np.random.default_rng(seed)
+    starts, counts = O.split_batch(w.B, w.G)
+    if integer:
+        return [rng.integers(-8, 9, size=(counts[r], w.T, w.dim)).astype(np.float32) for r in range(w.G)]
+    return [rng.standard_normal((counts[r], w.T, w.dim)).astype(np.float32) for r in range(w.G)]
+
+
+def test_bwd_bruteforce():
+    w = synth.make_workload("tiny", G=2, pmin=0, pmax=5, B=9, T=3, dim=4, rows=7)
+    offs, idxs = _csrs(w, 3)
+    dY = _dY(w, 1, integer=False)
+    dW, S, cnt = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    starts, counts = O.split_batch(w.B, w.G)
+    for t in range(w.T):
+        o = int(w.owner[t])
+        tl = list(w.local_tables(o)).index(t)
+        ref = [[0.0] * w.dim for _ in range(int(w.rows[t]))]
+        for b in range(w.B):
+            r = max(i for i in range(w.G) if starts[i] <= b)
+            lo, hi = int(offs[o][tl * w.B + b]), int(offs[o][tl * w.B + b + 1])
+            for j in range(lo, hi):
+                for k in range(w.dim):
+                    ref[int(idxs[o][j])][k] += float(dY[r][b - starts[r], t, k])
+        assert np.allclose(dW[t], np.array(ref), rtol=0, atol=1e-12)
+
+
+def test_bwd_adjoint_identity():
+    """<pool(W), dY> == <W, dW> : the backward is the exact transpose of the forward."""
+    w = synth.make_workload("tiny", G=3, mode="int", pmin=0, pmax=30, B=40, T=5, dim=8, rows=50)
+    tabs = _tables(w)
+    offs, idxs = _csrs(w, 8)
+    Y = O.emb_forward(tabs, w.owner, offs, idxs, w.B, w.G)
+    dY = _dY(w, 2)
+    dW, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    lhs = sum(float((Y[r].astype(np.float64) * dY[r]).sum()) for r in range(w.G))
+    rhs = sum(float((tabs[t].astype(np.float64) * dW[t]).sum()) for t in range(w.T))
+    assert lhs == rhs
+
+
+def test_bwd_matches_torch_autograd():
+    torch = pytest.importorskip("torch")
+    w = synth.make_workload("tiny", G=1, pmin=0, pmax=20, B=30, T=2, dim=8, rows=40)
+    tabs = _tables(w)
+    offs, idxs = _csrs(w, 4)
+    dY = _dY(w, 5, integer=False)
+    dW, _, cnt = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, 1)
+    for t in range(w.T):
+        o, lo, hi = O.rank_table_csr(offs[0], t, w.B)
+        Wt = torch.from_numpy(tabs[t].astype(np.float64)).requires_grad_(True)
+        y = torch.nn.functional.embedding_bag(torch.from_numpy(idxs[0][lo:hi]), Wt, torch.from_numpy(o[:-1]), mode="sum")
+        y.backward(torch.from_numpy(dY[0][:, t].astype(np.float64)))
+        assert np.allclose(Wt.grad.numpy(), dW[t], rtol=1e-12, atol=1e-12)
+        assert cnt[t].sum() == hi - lo
+
+
+def test_bwd_placement_invariance():
+    outs = []
+    for own in ([0, 0, 1, 1, 1], [1, 0, 1, 0, 1], [1, 1, 1, 1, 1]):
+        w = synth.make_workload("tiny", G=2, pmin=0, pmax=9, B=21, T=5, dim=4, rows=30, owner=np.array(own))
+        offs, idxs = _csrs(w, 6)
+        dW, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, _dY(w, 9), w.B, w.G)
+        outs.append(dW)
+    for d in outs[1:]:
+        for a, b in zip(d, outs[0]):
+            assert np.array_equal(a, b)
