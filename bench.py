@@ -41,6 +41,8 @@ def parse():
     p.add_argument("--config", default="weak")
     p.add_argument("--dist", default=None, help="override index distribution (zipf|uniform)")
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--mode", default="forward", choices=["forward", "backward"],
+                   help="backward = SURVEY row f2 (emb_backward: pull output gradients, scatter into dW)")
     p.add_argument("--batches", type=int, default=4, help="distinct pre-generated batches cycled")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
@@ -216,6 +218,70 @@ def reference_arm(args):
     return 0
 
 
+# ------------------------------------------------------------------------------ backward (f2)
+def run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq, nbags, remote_bags, barrier, timed):
+    """One step = publish this rank's output-gradient slot + the fused backward kernel
+    (one-sided loads of dY from the DP ranks, red.add into dW).  dY is synthetic
+    (standard normal, filled once per slot, untimed); dW accumulates across steps."""
+    import torch
+    import torch.distributed as dist
+    dW = [torch.zeros((int(w.rows[t]), w.dim), device=dev) for t in w.local_tables(rank)]
+    gen = torch.Generator(device=dev).manual_seed(1234 + rank)
+    for _ in range(2):                                    # fill both ring slots once (untimed)
+        with torch.cuda.stream(stream):
+            g = layer.grad_slot(stream)
+            g.normal_(generator=gen)
+        layer.grad_ready(stream)
+        o, x = batches[0]
+        layer.backward(o, x, dW, 0, stream, publish=False)
+    torch.cuda.synchronize()
+
+    def bwd(s):
+        o, x = batches[s % len(batches)]
+        layer.grad_slot(stream)                           # ring protocol (waits for peers' reads)
+        layer.backward(o, x, dW, 0, stream)
+
+    for s in range(args.warmup):
+        bwd(s)
+    barrier()
+    with ClockSampler(local) as clk:
+        ms = timed(bwd, args.steps)
+    assert layer.device_error() == 0, "device error during the timed region"
+    value = w.B / (ms * 1e-3)
+    e, row = 4, w.dim * 4                                 # dW and dY are fp32
+    nnz_m, uniq_m = float(np.mean(nnz)), float(np.mean(uniq))
+    lookup_bytes = nnz_m * (2 * row + 8) + nbags * (8 + row)      # row RMW per lookup + dY/offset per bag
+    comp_bytes = uniq_m * 2 * row + nnz_m * 8 + nbags * (8 + row)  # each touched dW row read+written once
+    nvl = remote_bags * row
+    peak, peak_kind = hbm_peak()
+    t_hbm, t_nvl = comp_bytes / (peak * 1e9), nvl / (NVLINK_GBS * 1e9)
+    bound = "hbm" if t_hbm >= t_nvl else "nvlink"
+    ach = (comp_bytes if bound == "hbm" else nvl) / (ms * 1e-3) / 1e9
+    pk = peak if bound == "hbm" else NVLINK_GBS
+    roof = {"bound": bound, "achieved": ach, "peak": pk, "unit": "GB/s", "frac": ach / pk, "traffic": None,
+            "kernel": "emb_bwd_kernel (one-sided dY loads + red.add.v4.f32 into dW)",
+            "algorithmic_bytes_per_launch": comp_bytes if bound == "hbm" else nvl,
+            "basis": "compulsory: each touched dW row read+written once (2*d*4) + every index + every offset + "
+                     "every dY vector read once",
+            "lookup_counted": {"bytes": lookup_bytes, "achieved": lookup_bytes / (ms * 1e-3) / 1e9,
+                               "frac": lookup_bytes / (ms * 1e-3) / 1e9 / peak},
+            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs", "t_roof_ms": max(t_hbm, t_nvl) * 1e3}
+    layer.close()
+    if N > 1:
+        dist.barrier()
+    if rank == 0:
+        line = {"metric": "EMB bwd samples/sec (max over ranks)", "value": value, "unit": "samples/s", "n_gpus": N,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None, "dtype": "f32",
+                "data": "synthetic", "config": {**config_desc(w, N), "mode": "backward (SURVEY f2)"},
+                "roofline": roof, "cpu_baseline": None, "e2e": None, "gpu_launches": args.steps * (2 if N > 1 else 1),
+                "clocks": clk.summary()}
+        print(json.dumps(line), flush=True)
+    if N > 1:
+        dist.destroy_process_group()
+    return 0
+
+
 # ------------------------------------------------------------------------------ GPU arm
 def main():
     args = parse()
@@ -257,7 +323,7 @@ def main():
         k, v = kv.split("=")
         opts[k] = int(v)
     layer = PgasEmbedding(rank, N, local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
-                          torch_allgather() if N > 1 else None, opts)
+                          torch_allgather() if N > 1 else None, opts, backward=(args.mode == "backward"))
     nnz = [int(b[0][-1].item()) for b in batches]
     uniq = [unique_rows(w, rank, b) for b in batches]     # untimed: compulsory-traffic basis
     T_r = len(w.local_tables(rank))
@@ -290,6 +356,10 @@ def main():
     def fwd(s):
         o, x = batches[s % len(batches)]
         layer.forward(o, x, 0, stream)
+
+    if args.mode == "backward":
+        return run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq, nbags, remote_bags,
+                            barrier, timed)
 
     for s in range(args.warmup):
         fwd(s)

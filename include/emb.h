@@ -95,7 +95,7 @@ emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_f
                       emb_ctx_t** out);
 
 /* Collective.  Describe ALL T tables and register this rank's local ones.
- *   rows[T]    : rows M_t of every table (host)
+ *   rows[T]    : rows M_t of every table (host), 1 <= M_t < 2^31
  *   owner[T]   : rank holding table t, in [0, world_size) (host)  -- table-wise MP (L99-101)
  *   dim        : embedding dim d; d*sizeof(weight) must be a multiple of 8 and either
  *                <= 512 bytes or a multiple of 512 bytes up to 4096

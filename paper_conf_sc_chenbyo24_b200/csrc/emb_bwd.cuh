@@ -120,38 +120,63 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
         while (b >= p.bstart[dst + 1]) ++dst;
         return p.gsrc[dst] + ((b - p.bstart[dst]) * p.T + tglob) * rowbytes + lane * VB;
       };
+      // Per bag: the bag's gradient vector (prefetched one bag ahead, with the bag's first
+      // 32 row ids) is added once per DISTINCT row of each 32-id slice, multiplied by the
+      // row's multiplicity (match.any): zipf-hot rows repeat inside a bag, and fewer
+      // atomics on the same L2 address is what bounds this kernel.
+      auto bag_start = [&](int bag) -> int64_t { return __shfl_sync(kFull, o_l, bag); };
+      auto load_ids = [&](int64_t from, int64_t to) -> uint32_t {
+        return (from + lane < to) ? (uint32_t)ld_stream_i64(p.indices + from + lane) : (0x80000000u | lane);
+      };
       uint32_t gn[NV][W];
-      if (active) {
-        const char* a = gaddr(0);
+      uint32_t xn = 0;
+      {
+        const int64_t s0 = bag_start(0), e0 = bag_start(1);
+        xn = load_ids(s0, e0);
+        if (active) {
+          const char* a = gaddr(0);
 #pragma unroll
-        for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
+          for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
+        }
       }
-      const int64_t pos0 = __shfl_sync(kFull, o_l, 0);
-      int64_t pos = pos0;
-      int64_t batch = -1;                                 // first position held in `my`
-      uint32_t my = 0;
       for (int bag = 0; bag < nb; ++bag) {
         uint32_t g[NV][W];
 #pragma unroll
         for (int v = 0; v < NV; ++v)
 #pragma unroll
           for (int i = 0; i < W; ++i) g[v][i] = gn[v][i];
-        if (bag + 1 < nb && active) {                     // next bag's gradient in flight
-          const char* a = gaddr(bag + 1);
-#pragma unroll
-          for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
-        }
-        const int64_t end = __shfl_sync(kFull, o_l, bag + 1);
-        for (; pos < end; ++pos) {
-          if (pos >= batch + 32 || batch < 0) {
-            batch = pos;
-            my = (pos + lane < __shfl_sync(kFull, o_l, nb)) ? (uint32_t)ld_stream_i64(p.indices + pos + lane) : 0u;
-          }
-          const uint32_t x = __shfl_sync(kFull, my, (int)(pos - batch));
+        uint32_t x = xn;
+        const int64_t s0 = bag_start(bag), e0 = bag_start(bag + 1);
+        if (bag + 1 < nb) {                               // next bag: gradient + first ids in flight
+          const int64_t s1 = e0, e1 = bag_start(bag + 2 > 31 ? 31 : bag + 2);
+          xn = load_ids(s1, bag + 1 < nb ? e1 : s1);
           if (active) {
-            char* rp = dwl + (uint64_t)x * (uint64_t)rowbytes;
+            const char* a = gaddr(bag + 1);
 #pragma unroll
-            for (int v = 0; v < NV; ++v) red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), g[v]);
+            for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
+          }
+        }
+        for (int64_t c0 = s0; c0 < e0; c0 += 32) {
+          if (c0 != s0) x = load_ids(c0, e0);
+          const unsigned same = __match_any_sync(kFull, x);
+          const bool lead = (x & 0x80000000u) == 0 && (__ffs(same) - 1) == lane;
+          unsigned leaders = __ballot_sync(kFull, lead);
+          const float mult = (float)__popc(same);
+          while (leaders) {
+            const int l = __ffs(leaders) - 1;
+            leaders &= leaders - 1;
+            const uint32_t xl = __shfl_sync(kFull, x, l);
+            const float m = __shfl_sync(kFull, mult, l);
+            if (active) {
+              char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
+#pragma unroll
+              for (int v = 0; v < NV; ++v) {
+                uint32_t gm[W];
+#pragma unroll
+                for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
+                red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), gm);
+              }
+            }
           }
         }
       }

@@ -241,7 +241,8 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   c->local.clear();
   for (int g = 0; g < kMaxG; ++g) c->tables_of[g].clear();
   for (int t = 0; t < num_tables; ++t) {
-    if (rows[t] < 1) FAIL(c, EMB_ERR_ARG, "rows[%d] = %lld < 1", t, (long long)rows[t]);
+    if (rows[t] < 1 || rows[t] > 0x7fffffffLL)
+      FAIL(c, EMB_ERR_ARG, "rows[%d] = %lld not in [1, 2^31) (row ids travel as 32-bit)", t, (long long)rows[t]);
     if (owner[t] < 0 || owner[t] >= c->G) FAIL(c, EMB_ERR_ARG, "owner[%d] = %d not in [0, %d)", t, owner[t], c->G);
     c->tables_of[owner[t]].push_back(t);
     if (owner[t] == c->rank) c->local.push_back(t);

@@ -79,3 +79,40 @@ def test_weak_config_uniform_sampled():
 @pytest.mark.slow
 def test_strong_config_g1_aliased_sampled():
     _sampled_parity("strong", 500)
+
+
+def test_weak_config_backward_sampled_rows():
+    """f2 at the weak config's full size: integer dY, sampled dW rows of two tables
+    recomputed by the oracle's definition from the regenerated CSR (exact)."""
+    w = synth.make_workload("weak", G=1)
+    seed = w.batch_seed(0)
+    tables, _ = SG.local_tables(w, 0, DEV)
+    off, idx = SG.rank_csr(w, seed, 0, DEV)
+    layer = PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype, backward=True)
+    check_t = [0, w.T - 1]
+    try:
+        dW = [torch.zeros((int(w.rows[t]), w.dim), device=DEV) if t in check_t else
+              torch.zeros((1, w.dim), device=DEV) for t in range(w.T)]
+        # tables not checked still need a full-size dW: reuse one scratch buffer for them
+        scratch = torch.zeros((int(w.rows[1]), w.dim), device=DEV)
+        dW = [d if t in check_t else scratch for t, d in enumerate(dW)]
+        rng = np.random.default_rng(3)
+        dY = rng.integers(-8, 9, size=(w.B, w.T, w.dim)).astype(np.float32)
+        g = layer.grad_slot()
+        g.copy_(torch.from_numpy(dY).to(DEV))
+        layer.backward(off, idx, dW)
+        torch.cuda.synchronize()
+        assert layer.device_error() == 0
+        for t in check_t:
+            o, x = synth.table_csr(w, seed, t)
+            bag_of = np.repeat(np.arange(w.B), np.diff(o))
+            rows = np.unique(np.concatenate([x[:50], rng.integers(0, int(w.rows[t]), 50)]))
+            got = dW[t][torch.from_numpy(rows).to(DEV)].cpu().numpy()
+            for i, r in enumerate(rows):
+                sel = bag_of[x == r]
+                ref = dY[sel, t].astype(np.float64).sum(axis=0) if sel.size else np.zeros(w.dim)
+                assert np.array_equal(got[i].astype(np.float64), ref), (t, r)
+    finally:
+        layer.close()
+        del tables
+        torch.cuda.empty_cache()

@@ -87,3 +87,74 @@ def test_cross_process_ipc_pgas(G, flags, owner):
         assert tb == "", tb
         assert ok, f"rank {rank} output != oracle"
         assert err == 0, f"rank {rank} device error {err}"
+
+
+def _bwd_worker(rank, G, port, q, epochs):
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    try:
+        import torch.distributed as dist
+
+        import emb_test_helpers as H
+        import synth
+        from oracle import emb_oracle as O
+        from paper_conf_sc_chenbyo24_b200.comm import torch_allgather
+        from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
+
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=G)
+        w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=97, T=6, dim=64, rows=400, dist="zipf")
+        tabs = H.np_tables(w)
+        dev = torch.device("cuda", 0)
+        local = [torch.from_numpy(tabs[int(w.phys[t])]).to(dev) for t in w.local_tables(rank)]
+        layer = PgasEmbedding(rank, G, 0, w.rows, w.owner, w.dim, local, w.B, "f32", "f32", torch_allgather(),
+                              {"timeout_ms": 20000}, backward=True)
+        dW = [torch.zeros((int(w.rows[t]), w.dim), device=dev) for t in w.local_tables(rank)]
+        rng = np.random.default_rng(77)
+        _, counts = O.split_batch(w.B, G)
+        dYs_all = [[rng.integers(-8, 9, size=(counts[r], w.T, w.dim)).astype(np.float32) for r in range(G)]
+                   for _ in range(epochs)]
+        o, x = synth.rank_csr(w, 55, rank)
+        od, xd = torch.from_numpy(o).to(dev), torch.from_numpy(x).to(dev)
+        s = torch.cuda.Stream()
+        for ep in range(epochs):
+            with torch.cuda.stream(s):
+                g = layer.grad_slot(s)
+                g.copy_(torch.from_numpy(dYs_all[ep][rank]).to(dev))
+            layer.backward(od, xd, dW, 0, s)          # one rank per process: publish + compute
+        s.synchronize()
+        offs, idxs = zip(*[synth.rank_csr(w, 55, r) for r in range(G)])
+        ok = True
+        acc = None
+        for ep in range(epochs):
+            ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dYs_all[ep], w.B, G)
+            acc = ref if acc is None else [a + b for a, b in zip(acc, ref)]
+        for tl, t in enumerate(w.local_tables(rank)):
+            ok = ok and np.array_equal(dW[tl].cpu().numpy().astype(np.float64), acc[int(t)])
+        err = layer.device_error()
+        layer.close()
+        dist.destroy_process_group()
+        q.put((rank, bool(ok), int(err), ""))
+    except Exception:
+        import traceback
+        q.put((rank, False, -1, traceback.format_exc()))
+
+
+@pytest.mark.parametrize("G", [2, 3])
+def test_cross_process_ipc_backward(G):
+    """f2 over real IPC: 4 epochs reuse both grad slots (ready/done flag ring)."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_bwd_worker, args=(r, G, port, q, 4)) for r in range(G)]
+    for p in ps:
+        p.start()
+    res = sorted(q.get(timeout=240) for _ in range(G))
+    for p in ps:
+        p.join(timeout=60)
+    for rank, ok, err, tb in res:
+        assert tb == "", tb
+        assert ok, f"rank {rank} dW != oracle"
+        assert err == 0, f"rank {rank} device error {err}"
