@@ -4,8 +4,12 @@
 namespace emb {
 namespace {
 template <int VB, int NV, typename WT, typename OT, bool CHECK>
-KernelFn pick_u(int unroll, int mb, bool full) {
+KernelFn pick_u(int unroll, int mb, bool full, bool sidx) {
   if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 4, false>;  // rows narrower than a warp
+  if constexpr (!CHECK && NV == 1) {
+    if (sidx && unroll == 4 && mb == 4) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, true>;
+    if (sidx && unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, false, 6, true, true>;
+  }
   if (unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, CHECK, 6, true>;
   switch (mb) {
     case 1: return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 1, true>;
@@ -14,7 +18,7 @@ KernelFn pick_u(int unroll, int mb, bool full) {
   }
 }
 template <int VB, int NV, typename WT, typename OT>
-KernelFn pick_c(int unroll, bool check, int mb, bool full) {
+KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx) {
   if (unroll >= 8) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
     if constexpr (NV == 1) {
       if (unroll == 16)
@@ -23,19 +27,20 @@ KernelFn pick_c(int unroll, bool check, int mb, bool full) {
     }
     unroll = 4;
   }
-  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full) : pick_u<VB, NV, WT, OT, false>(unroll, mb, full);
+  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full, sidx)
+               : pick_u<VB, NV, WT, OT, false>(unroll, mb, full, sidx);
 }
 }  // namespace
 
-KernelFn pick_tile_f32_bf16(int vb, int nv, int unroll, bool check, int mb, bool full) {
+KernelFn pick_tile_f32_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx) {
   using WT = float;
   using OT = __nv_bfloat16;
-  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full);
+  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full, sidx);
   switch (nv) {
-    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full);
-    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full);
-    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full);
-    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full);
+    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full, sidx);
+    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full, sidx);
+    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full, sidx);
+    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx);
   }
 }
 }  // namespace emb

@@ -84,7 +84,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0;  // 0: auto per tile
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -144,17 +144,19 @@ static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb 
 static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
 static size_t dyn_smem(const emb_ctx* c) {
-  return (eff_unroll(c) >= 8 && c->nv == 1) ? (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb : 0;
+  if (eff_unroll(c) >= 8 && c->nv == 1) return (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb;
+  if (c->sidx && c->nv == 1 && full_row(c)) return (size_t)(kBlock / 32) * 1024;  // id ring: 4 x 32 x 8 B per warp
+  return 0;
 }
 
 // ---------------------------------------------------------------------------- kernel dispatch
 namespace {
 
-KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full) {
-  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full);
-  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full);
-  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full);
-  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full);
+KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx) {
+  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx);
+  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx);
+  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx);
+  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx);
 }
 
 // row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
@@ -411,7 +413,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 }
 
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c));
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0);
   const size_t smem = dyn_smem(c);
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = c->ctas_per_sm;
@@ -724,7 +726,7 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   i->epoch = c->epoch;
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0 && c->registered) {
-    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c));
+    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), c->sidx != 0);
     const size_t smem = dyn_smem(c);
     if (smem > 0) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem);
@@ -751,6 +753,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     if (v != 0 && v != 1 && v != 4 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4 or 6");
     c->minblocks = (int)v;
   }
+  else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
   else if (!strcmp(key, "enable_backward")) {
     if (c->registered) FAIL(c, EMB_ERR_STATE, "enable_backward must be set before emb_register_tables");
     c->bwd_enabled = v != 0;
