@@ -164,7 +164,11 @@ class OracleSampler:
         self.lt = list(w.local_tables(rank))
         t0 = self.lt[0]
         self.W = synth.table_rows(w.table_seed, int(w.phys[t0]), int(w.rows[t0]), w.dim, w.mode, w.wdtype)
-        self.csrs = [synth.table_csr(w, w.batch_seed(0), int(t)) for t in self.lt[:max_tables]]
+        M0 = int(w.rows[t0])
+        self.folded = any(int(w.rows[t]) != M0 for t in self.lt[:max_tables])
+        # mixed table sizes (large config): fold the sampled tables' ids into the one
+        # physical table generated for timing (values do not change the oracle's work)
+        self.csrs = [(o, x % M0) for o, x in (synth.table_csr(w, w.batch_seed(0), int(t)) for t in self.lt[:max_tables])]
 
     def run(self, budget_s=12.0, min_tables=1):
         O, w = self.O, self.w
@@ -180,7 +184,8 @@ class OracleSampler:
         per_rank_s = dt * len(self.lt) / done
         return {"value": w.B / per_rank_s, "unit": "samples/s", "cores": 1, "kind": "oracle",
                 "sample": f"{done} of {len(self.lt)} local tables x full batch {w.B} ({lookups} lookups; table values "
-                          f"from one physical {int(w.rows[self.lt[0]])}x{w.dim} table) + MP->DP layout, {dt:.2f}s, "
+                          f"from one physical {int(w.rows[self.lt[0]])}x{w.dim} table{', ids folded into it' if self.folded else ''}) "
+                          f"+ MP->DP layout, {dt:.2f}s, "
                           f"extrapolated to the rank's workload by table count",
                 "seconds": dt, "rank_seconds": per_rank_s}
 

@@ -218,7 +218,8 @@ class Workload:
         return d
 
     def batch_seed(self, batch_id: int) -> int:
-        cid = {"tiny": 0, "single": 1, "weak": 2, "weak_paper": 2, "strong": 3, "large": 4}.get(self.name, 9)
+        cid = {"tiny": 0, "single": 1, "weak": 2, "weak_paper": 2, "strong": 3, "large": 4,
+               "large_shard": 4}.get(self.name, 9)
         return 20241119 + 1000 * cid + int(batch_id)
 
     def elem_bytes(self) -> int:
@@ -278,6 +279,10 @@ def make_workload(name: str, G: int = 1, *, dist: Optional[str] = None, mode: st
         kw = dict(T=208, rows=2_000_000, dim=128, B=65536, pmin=1, pmax=32, dist="zipf", wdtype="f32", odtype="f32")
     elif name == "large":
         kw = dict(T=512, rows=large_rows(512), dim=256, B=65536, pmin=1, pmax=100, dist="zipf", wdtype="bf16", odtype="bf16")
+    elif name == "large_shard":   # one rank's LPT share of `large` (64 tables, 150 GB bf16) run at G = 1
+        share = large_rows(512)[lpt_placement(large_rows(512), 8) == 0]
+        kw = dict(T=len(share), rows=share, dim=256, B=65536, pmin=1, pmax=100, dist="zipf", wdtype="bf16",
+                  odtype="bf16")
     else:
         raise ValueError(name)
     kw.update(over)
