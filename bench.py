@@ -383,12 +383,23 @@ def main():
     achieved = (hbm_bytes if bound == "hbm" else nvl_bytes) / (ms * 1e-3) / 1e9
     pk = peak if bound == "hbm" else NVLINK_GBS
     traffic = None
+    l2 = None
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             tj = json.load(f)
         key = f"{w.name}:{w.dist}:G{N}"  # profiles/traffic.json: ncu --set full of this workload
         if key in tj:
             traffic = tj[key]["dram_bytes_per_launch"]
+            with open(os.path.join(ROOT, "profiles", "l2_probe.json")) as f:
+                l2_peak = float(json.load(f)["l2_read_peak_gbs"])
+            l2_bytes = tj[key].get("l2_read_bytes_per_launch")
+            if l2_bytes:
+                # second roof: L2->SM read traffic of this kernel (ncu) over the measured L2
+                # streaming read bandwidth (tools/l2_probe.py); binds under zipf reuse
+                l2 = {"bytes": l2_bytes, "achieved": l2_bytes / (ms * 1e-3) / 1e9, "peak": l2_peak, "unit": "GB/s",
+                      "frac": l2_bytes / (ms * 1e-3) / 1e9 / l2_peak,
+                      "source": "ncu lts__t_sectors_srcunit_tex_op_read x 32 B (profiles/traffic.json) / "
+                                "profiles/l2_probe.json"}
     except Exception:
         pass
     roof = {"bound": bound, "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": achieved / pk,
@@ -402,7 +413,8 @@ def main():
                                        "because L1/L2 serve repeated rows"},
             "unique_rows_per_batch": float(np.mean(uniq)), "lookups_per_batch": float(np.mean(nnz)),
             "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else "measured peer copy 770 GB/s (B200_PROFILING.md)",
-            "t_roof_ms": max(t_hbm, t_nvl) * 1e3, "frac_of_roofline_time": max(t_hbm, t_nvl) * 1e3 / ms}
+            "t_roof_ms": max(t_hbm, t_nvl) * 1e3, "frac_of_roofline_time": max(t_hbm, t_nvl) * 1e3 / ms,
+            "l2": l2}
 
     extra = {}
     # ---- uniform-index control (lookup bytes ~= DRAM bytes; no zipf reuse)

@@ -21,6 +21,8 @@ WANT = {
     "launch__block_size": "block",
     "smsp__inst_executed.sum": "inst",
     "sm__cycles_elapsed.avg.per_second": "sm_hz",
+    "lts__t_sectors_srcunit_tex_op_read.sum": "l2_read_sectors",
+    "lts__t_sectors_srcunit_tex_lookup_miss.sum": "l2_miss_sectors",
 }
 
 
@@ -52,6 +54,10 @@ def summary(path):
                 elif u == "ns":
                     v *= 1e-9
                 d[name] = v
+        if "l2_read_sectors" in d:
+            d["l2_read_bytes"] = d["l2_read_sectors"] * 32
+            if "duration" in d:
+                d["l2_read_gbs"] = d["l2_read_bytes"] / d["duration"] / 1e9
         if "dram_read" in d and "duration" in d:
             d["dram_gbs"] = (d["dram_read"] + d.get("dram_write", 0)) / d["duration"] / 1e9
         res.append(d)

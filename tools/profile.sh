@@ -11,3 +11,5 @@ ncu --set full --clock-control none --import-source on -k regex:emb_fwd_kernel -
 ncu --set full --clock-control none --import-source on -k regex:emb_fwd_kernel -s 3 -c 1 -o $OUT/full_weak_uniform -f $BENCH --dist uniform > $OUT/full_uniform.log 2>&1
 ncu --set full --clock-control none --import-source on -k regex:emb_fwd_kernel -s 3 -c 1 -o $OUT/full_single_zipf -f $BENCH --config single > $OUT/full_single.log 2>&1
 ls -la $OUT
+# f2 backward (zipf)
+ncu --set full --clock-control none --import-source on -k regex:emb_bwd_kernel -s 3 -c 1 -o $OUT/full_weak_zipf_backward -f $BENCH --mode backward > $OUT/full_bwd.log 2>&1

@@ -28,14 +28,16 @@ def main():
     ap.add_argument("--opts", nargs="*", default=[""])
     ap.add_argument("--baseline", action="store_true")
     ap.add_argument("--repeat", type=int, default=1)
+    ap.add_argument("--rows", type=int, default=None, help="override rows per table (e.g. an L2-resident table)")
     a = ap.parse_args()
     dev = torch.device("cuda", 0)
-    w = synth.make_workload(a.config, G=1)
+    over = {"rows": a.rows} if a.rows else {}
+    w = synth.make_workload(a.config, G=1, **over)
     tables, _ = SG.local_tables(w, 0, dev)
     layer = PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype)
     s = torch.cuda.Stream()
     for dist in a.dists.split(","):
-        wd = synth.make_workload(a.config, G=1, dist=dist)
+        wd = synth.make_workload(a.config, G=1, dist=dist, **over)
         bs = [SG.rank_csr(wd, wd.batch_seed(i), 0, dev) for i in range(3)]
         nnz = np.mean([int(b[0][-1]) for b in bs])
         byt = nnz * (w.dim * w.elem_bytes() + 8) + w.T * w.B * (8 + w.dim * w.out_elem_bytes())
@@ -67,7 +69,7 @@ def main():
                 clk = pw = None
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / a.steps
-            print(json.dumps({"config": a.config, "dist": dist, "opts": o, "ms": round(ms, 4),
+            print(json.dumps({"config": a.config, "rows": int(w.rows[0]), "dist": dist, "opts": o, "ms": round(ms, 4),
                               "Msamples_s": round(w.B / ms / 1e3, 3), "GBs": round(byt / ms / 1e6, 1),
                               "sm_mhz": clk, "power_w": pw}), flush=True)
             assert layer.device_error() == 0
