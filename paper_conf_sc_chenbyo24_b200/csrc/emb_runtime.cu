@@ -84,7 +84,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 0;  // 0: auto per tile
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 0, carveout = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -416,6 +416,9 @@ static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags,
   KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0);
   const size_t smem = dyn_smem(c);
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
+  // carve-out that fits (the rest of the 256 KB per SM becomes L1)
+  if (c->carveout >= 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, c->carveout));
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0) {
     CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem));
@@ -754,6 +757,10 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->minblocks = (int)v;
   }
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
+  else if (!strcmp(key, "carveout")) {
+    if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");
+    c->carveout = (int)v;
+  }
   else if (!strcmp(key, "enable_backward")) {
     if (c->registered) FAIL(c, EMB_ERR_STATE, "enable_backward must be set before emb_register_tables");
     c->bwd_enabled = v != 0;
