@@ -46,7 +46,7 @@ import numpy as np
 __all__ = [
     "validate_csr", "pool_table_f32", "pool_table_f64", "rne_bf16", "bf16_to_f32",
     "split_batch", "rank_table_csr", "mp_to_dp", "emb_forward", "pool_bag_f32",
-    "pool_bag_f64", "s_normalized_error", "emb_backward",
+    "pool_bag_f64", "s_normalized_error", "emb_backward", "emb_forward_sharded",
 ]
 
 
@@ -240,3 +240,48 @@ def emb_backward(rows: Sequence[int], dim: int, owner: Sequence[int], rank_offse
             np.add.at(S[t], x, np.abs(g))
             np.add.at(cnt[t], x, 1)
     return dW, S, cnt
+
+
+# ----------------------------------------------------------------------------- row-wise sharding (f3)
+def emb_forward_sharded(tables: Sequence[np.ndarray], shards: Sequence[Tuple[int, int, int, int, int]],
+                        rank_offsets: Sequence[np.ndarray], rank_indices: Sequence[np.ndarray], B: int, G: int,
+                        out_dtype: str = "f32") -> List[np.ndarray]:
+    """Row-wise sharded forward (§V: "partitioning by rows ... merge the sparse
+    input partitioning into the computation kernel").
+
+    shards: (t, s, lo, hi, owner) -- shard s of table t holds rows [lo, hi) on rank `owner`;
+    a table with one shard (lo = 0, hi = M_t) is table-wise.  Each rank's CSR lists its
+    local shards in ascending (t, s) order, each with the FULL bag list of table t and
+    GLOBAL row ids (the partitioning happens in the kernel).  Definition:
+      partial_{t,s}[b] = sum, in CSR order from the first kept row, of W_t[x] over the
+                         bag's ids with lo <= x < hi (+0.0 if none)            (C4, C2)
+      Z_t[b]           = partial_{t,0}[b] + partial_{t,1}[b] + ... in shard order (float32)
+    then the usual layout conversion Y_r[i, t] = Z_t[s_r + i] (C8, C9)."""
+    T = len(tables)
+    by_t: Dict[int, list] = {}
+    for (t, s, lo, hi, o) in shards:
+        by_t.setdefault(int(t), []).append((int(s), int(lo), int(hi), int(o)))
+    partial: Dict[Tuple[int, int], np.ndarray] = {}
+    for r in range(G):
+        local = sorted((int(t), int(s), int(lo), int(hi)) for (t, s, lo, hi, o) in shards if int(o) == r)
+        for k, (t, s, lo, hi) in enumerate(local):
+            o, a, b = rank_table_csr(rank_offsets[r], k, B)
+            x = np.asarray(rank_indices[r][a:b], dtype=np.int64)
+            validate_csr(o, x, int(np.asarray(tables[t]).shape[0]))
+            keep = (x >= lo) & (x < hi)
+            # re-pack the bag list with only the kept ids, preserving CSR order
+            ck = np.concatenate([[0], np.cumsum(keep.astype(np.int64))])
+            kept_per_bag = ck[o[1:]] - ck[o[:-1]]
+            o2 = np.zeros(B + 1, dtype=np.int64)
+            np.cumsum(kept_per_bag, out=o2[1:])
+            W = np.asarray(tables[t], dtype=np.float32)
+            partial[(t, s)] = pool_table_f32(W, o2, x[keep])
+    Z = []
+    for t in range(T):
+        parts = sorted(by_t[t])
+        acc = partial[(t, parts[0][0])].copy()
+        for (s, _, _, _) in parts[1:]:
+            acc = acc + partial[(t, s)]
+        Z.append(acc)
+    Ys = mp_to_dp(Z, G)
+    return [rne_bf16(Y) for Y in Ys] if out_dtype == "bf16" else Ys

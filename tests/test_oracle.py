@@ -406,3 +406,80 @@ def test_bwd_placement_invariance():
     for d in outs[1:]:
         for a, b in zip(d, outs[0]):
             assert np.array_equal(a, b)
+
+
+# ------------------------------------------------------------------------------- row-wise sharding (f3)
+def _sharded_inputs(w, seed, shards):
+    """Per rank: for each local shard (ascending (t, s)) the FULL CSR of table t."""
+    offs, idxs = [], []
+    for r in range(w.G):
+        local = sorted((t, s) for (t, s, lo, hi, o) in shards if o == r)
+        oo, xx, base = [np.zeros(1, np.int64)], [], 0
+        for (t, s) in local:
+            o, x = synth.table_csr(w, seed, t)
+            oo.append(o[1:] + base)
+            xx.append(x)
+            base += int(o[-1])
+        offs.append(np.concatenate(oo))
+        idxs.append(np.concatenate(xx) if xx else np.zeros(0, np.int64))
+    return offs, idxs
+
+
+def _even_shards(w, nshard_of, owners_of):
+    sh = []
+    for t in range(w.T):
+        S = nshard_of(t)
+        cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(int)
+        for s in range(S):
+            sh.append((t, s, int(cuts[s]), int(cuts[s + 1]), owners_of(t, s)))
+    return sh
+
+
+def test_f3_single_shard_equals_tablewise():
+    w = synth.make_workload("tiny", G=2, pmin=0, pmax=20, B=33, T=4, dim=8, rows=200)
+    tabs = _tables(w)
+    shards = [(t, 0, 0, int(w.rows[t]), int(w.owner[t])) for t in range(w.T)]
+    offs, idxs = _sharded_inputs(w, 4, shards)
+    Ys = O.emb_forward_sharded(tabs, shards, offs, idxs, w.B, w.G)
+    o2, x2 = _csrs(w, 4)
+    Y = O.emb_forward(tabs, w.owner, o2, x2, w.B, w.G)
+    for a, b in zip(Ys, Y):
+        assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+
+
+def test_f3_integer_exact_and_bruteforce():
+    w = synth.make_workload("tiny", G=3, mode="int", pmin=0, pmax=40, B=29, T=3, dim=4, rows=90)
+    tabs = _tables(w)
+    shards = _even_shards(w, lambda t: t + 1, lambda t, s: (t + s) % 3)
+    offs, idxs = _sharded_inputs(w, 7, shards)
+    Ys = O.emb_forward_sharded(tabs, shards, offs, idxs, w.B, w.G)
+    starts, counts = O.split_batch(w.B, w.G)
+    for r in range(w.G):
+        for i in range(counts[r]):
+            b = starts[r] + i
+            for t in range(w.T):
+                o, x = synth.table_csr(w, 7, t)
+                ref = sum((tabs[t][int(v)].astype(np.float64) for v in x[o[b]:o[b + 1]]), np.zeros(w.dim))
+                assert np.array_equal(Ys[r][i, t].astype(np.float64), ref)
+
+
+def test_f3_shard_order_sum_and_tolerance():
+    """Float data: the sharded result is the shard-order sum of canonical partials (not the
+    unsharded canonical order) and stays within the S-normalised 1e-6 of the fp64 sum."""
+    w = synth.make_workload("tiny", G=2, pmin=1, pmax=100, B=40, T=2, dim=16, rows=500)
+    tabs = _tables(w)
+    shards = _even_shards(w, lambda t: 4, lambda t, s: s % 2)
+    offs, idxs = _sharded_inputs(w, 9, shards)
+    Ys = np.concatenate(O.emb_forward_sharded(tabs, shards, offs, idxs, w.B, w.G))
+    for t in range(w.T):
+        o, x = synth.table_csr(w, 9, t)
+        z64, S = O.pool_table_f64(tabs[t], o, x)
+        assert O.s_normalized_error(Ys[:, t], z64, S) <= 1e-6
+        cuts = np.linspace(0, int(w.rows[t]), 5).astype(int)
+        for b in range(w.B):
+            xb = x[o[b]:o[b + 1]]
+            parts = [O.pool_bag_f32(tabs[t][xb[(xb >= cuts[s]) & (xb < cuts[s + 1])]]) for s in range(4)]
+            acc = parts[0]
+            for p_ in parts[1:]:
+                acc = acc + p_
+            assert np.array_equal(acc.view(np.uint32), Ys[b, t].view(np.uint32))
