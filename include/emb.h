@@ -113,6 +113,26 @@ emb_status_t emb_register_tables(emb_ctx_t* ctx, int32_t num_tables, const int64
                                  int32_t dim, emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
                                  const void* const* local_weights);
 
+/* Collective.  f3 (§V "partitioning by rows ... merge the
+ * sparse input partitioning into the computation kernel"): like emb_register_tables but
+ * every table t is split into num_shards[t] contiguous row ranges.  shard_owner[] and
+ * shard_row_start[] list the shards of table 0, then table 1, ... (sum(num_shards)
+ * entries); shard s of t holds global rows [shard_row_start, next start or rows[t]) on
+ * rank shard_owner (first start 0, strictly increasing).  A table with one shard is
+ * table-wise.  local_weights[] lists this rank's shards in ascending (t, s), each pointing
+ * at the shard's first row.  The CSR passed to emb_forward lists, for every local shard
+ * in the same order, the FULL bag list of its table with GLOBAL row ids; the kernel skips
+ * other shards' ids (in-kernel partitioning), stores each bag's fp32 partial sum into the
+ * owner's partial slot (one-sided, like the pooled vectors), and after the exchange a
+ * combine kernel sums the partials in shard order into Y_r (bf16 out: RNE once).  Not
+ * supported with row-sharded tables: EMB_FWD_CHECK_BOUNDS, the comparison path,
+ * backward.  Errors as emb_register_tables. */
+emb_status_t emb_register_sharded_tables(emb_ctx_t* ctx, int32_t num_tables, const int64_t* rows,
+                                         const int32_t* num_shards, const int32_t* shard_owner,
+                                         const int64_t* shard_row_start, int32_t dim, emb_dtype_t weight_dtype,
+                                         emb_dtype_t out_dtype, int64_t global_batch,
+                                         const void* const* local_weights);
+
 /* Collective, stream-ordered, asynchronous: the fused PGAS forward (Listing 2).
  *   offsets : device int64[T_r*B + 1], table-major CSR: bag (t_l, b) spans
  *             indices[offsets[t_l*B+b] .. offsets[t_l*B+b+1]) (C11; L212-215)

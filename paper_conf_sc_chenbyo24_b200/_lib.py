@@ -37,6 +37,9 @@ SIGNATURES = {
     "emb_init": (C.c_int, [C.c_int, C.c_int, C.c_int, ALLGATHER_FN, C.c_void_p, C.POINTER(C.c_void_p)]),
     "emb_register_tables": (C.c_int, [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32), C.c_int32,
                                       C.c_int, C.c_int, C.c_int64, C.POINTER(C.c_void_p)]),
+    "emb_register_sharded_tables": (C.c_int, [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32),
+                                              C.POINTER(C.c_int32), C.POINTER(C.c_int64), C.c_int32, C.c_int, C.c_int,
+                                              C.c_int64, C.POINTER(C.c_void_p)]),
     "emb_forward": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(C.c_void_p)]),
     "emb_wait": (C.c_int, [C.c_void_p, C.c_void_p]),
     "emb_forward_host": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),

@@ -4,7 +4,15 @@
 namespace emb {
 namespace {
 template <int VB, int NV, typename WT, typename OT, bool CHECK>
-KernelFn pick_u(int unroll, int mb, bool full, bool sidx) {
+KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard) {
+  if constexpr (!CHECK) {
+    if (shard) {  // f3: row-sharded tables (in-kernel id partitioning, partial slots)
+      if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, false, false, true>;
+      if (unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, false, 6, true, false, true>;
+      if (NV > 1) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 1, true, false, true>;
+      return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, false, true>;
+    }
+  }
   if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 4, false>;  // rows narrower than a warp
   if constexpr (!CHECK && NV == 1) {
     if (sidx && unroll == 4 && mb == 4) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, true>;
@@ -18,8 +26,8 @@ KernelFn pick_u(int unroll, int mb, bool full, bool sidx) {
   }
 }
 template <int VB, int NV, typename WT, typename OT>
-KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx) {
-  if (unroll >= 8) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
+KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx, bool shard) {
+  if (unroll >= 8 && !shard) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
     if constexpr (NV == 1) {
       if (unroll == 16)
         return check ? emb_fwd_async_kernel<VB, NV, WT, OT, 16, true, 3> : emb_fwd_async_kernel<VB, NV, WT, OT, 16, false, 3>;
@@ -27,20 +35,20 @@ KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx) {
     }
     unroll = 4;
   }
-  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full, sidx)
-               : pick_u<VB, NV, WT, OT, false>(unroll, mb, full, sidx);
+  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full, sidx, shard)
+               : pick_u<VB, NV, WT, OT, false>(unroll, mb, full, sidx, shard);
 }
 }  // namespace
 
-KernelFn pick_tile_bf16_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx) {
+KernelFn pick_tile_bf16_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard) {
   using WT = __nv_bfloat16;
   using OT = __nv_bfloat16;
-  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full, sidx);
+  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full, sidx, shard);
   switch (nv) {
-    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full, sidx);
-    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full, sidx);
-    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full, sidx);
-    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx);
+    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full, sidx, shard);
+    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full, sidx, shard);
+    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full, sidx, shard);
+    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx, shard);
   }
 }
 }  // namespace emb

@@ -41,6 +41,8 @@ struct PeerBlob {
   uint64_t slot_bytes;   // bytes per slot (B_r*T*d*e_o rounded up to 256)
   uint64_t grad_off;     // byte offset of backward grad slot 0 (0 = backward not enabled)
   uint64_t gslot_bytes;  // bytes per grad slot (B_r*T*d*4 rounded up)
+  uint64_t part_off;     // f3: byte offset of partial slot 0 (0 = no row-sharded table)
+  uint64_t pslot_bytes;  // f3: bytes per partial slot
   int32_t device;
   int32_t pad;
   cudaIpcMemHandle_t handle;
@@ -72,7 +74,14 @@ struct emb_ctx {
   std::vector<int64_t> rows;
   std::vector<int32_t> owner;
   std::vector<int64_t> bstart;          // G+1
-  std::vector<int32_t> local;           // global ids of local tables
+  std::vector<int32_t> local;           // global table id of each local shard (ascending (t, s))
+  // f3 row-wise sharding
+  bool has_shard = false;
+  int T_sh = 0, S_max = 1;
+  size_t part_off = 0, pslot_bytes = 0;
+  std::vector<uint64_t> peer_part_off, peer_pslot_bytes;
+  int32_t* d_comb_tglob = nullptr;
+  int32_t* d_comb_nsh = nullptr;
   std::vector<int32_t> tables_of[kMaxG];
   TableDesc* d_tables = nullptr;
   // symmetric buffer (flags at offset 0, slots after)
@@ -152,11 +161,11 @@ static size_t dyn_smem(const emb_ctx* c) {
 // ---------------------------------------------------------------------------- kernel dispatch
 namespace {
 
-KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx) {
-  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx);
-  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx);
-  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx);
-  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx);
+KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard = false) {
+  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx, shard);
+  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx, shard);
+  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx, shard);
+  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx, shard);
 }
 
 // row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
@@ -211,12 +220,14 @@ emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_f
   return EMB_OK;
 }
 
-emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t* rows, const int32_t* owner,
-                                 int32_t dim, emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
-                                 const void* const* local_weights) {
+static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_t* rows, const int32_t* num_shards,
+                                  const int32_t* shard_owner, const int64_t* shard_row_start, int32_t dim,
+                                  emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
+                                  const void* const* local_weights) {
   if (!c) return EMB_ERR_ARG;
   if (c->registered) FAIL(c, EMB_ERR_STATE, "tables already registered");
-  if (num_tables < 1 || !rows || !owner) FAIL(c, EMB_ERR_ARG, "num_tables/rows/owner invalid");
+  if (num_tables < 1 || !rows || !num_shards || !shard_owner || !shard_row_start)
+    FAIL(c, EMB_ERR_ARG, "num_tables/rows/shards invalid");
   if (weight_dtype != EMB_F32 && weight_dtype != EMB_BF16) FAIL(c, EMB_ERR_ARG, "bad weight dtype");
   if (out_dtype != EMB_F32 && out_dtype != EMB_BF16) FAIL(c, EMB_ERR_ARG, "bad out dtype");
   if (global_batch < c->G) FAIL(c, EMB_ERR_ARG, "global_batch %lld < world_size %d", (long long)global_batch, c->G);
@@ -239,16 +250,47 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   c->vb = vb;
   c->nv = nv;
   c->rows.assign(rows, rows + num_tables);
-  c->owner.assign(owner, owner + num_tables);
+  c->owner.assign(num_tables, -1);
   c->local.clear();
   for (int g = 0; g < kMaxG; ++g) c->tables_of[g].clear();
+  // shards: (t, s) -> rows [lo, hi) on shard_owner; a table with one shard is table-wise
+  struct LocalShard { int t, s, part; int64_t lo, hi; };
+  std::vector<LocalShard> lsh;
+  std::vector<int32_t> comb_tglob, comb_nsh;
+  c->T_sh = 0;
+  c->S_max = 1;
+  for (int t = 0; t < num_tables; ++t)
+    if (num_shards[t] > 1) { ++c->T_sh; c->S_max = std::max(c->S_max, (int)num_shards[t]); }
+  int64_t k = 0;
+  int ksh = 0;
   for (int t = 0; t < num_tables; ++t) {
     if (rows[t] < 1 || rows[t] > 0x7fffffffLL)
       FAIL(c, EMB_ERR_ARG, "rows[%d] = %lld not in [1, 2^31) (row ids travel as 32-bit)", t, (long long)rows[t]);
-    if (owner[t] < 0 || owner[t] >= c->G) FAIL(c, EMB_ERR_ARG, "owner[%d] = %d not in [0, %d)", t, owner[t], c->G);
-    c->tables_of[owner[t]].push_back(t);
-    if (owner[t] == c->rank) c->local.push_back(t);
+    const int S = num_shards[t];
+    if (S < 1 || S > 64) FAIL(c, EMB_ERR_ARG, "num_shards[%d] = %d not in [1, 64]", t, S);
+    if (S > 1) {
+      comb_tglob.push_back(t);
+      comb_nsh.push_back(S);
+    }
+    for (int sh = 0; sh < S; ++sh, ++k) {
+      const int32_t o = shard_owner[k];
+      const int64_t lo = shard_row_start[k];
+      const int64_t hi = (sh + 1 < S) ? shard_row_start[k + 1] : rows[t];
+      if (o < 0 || o >= c->G) FAIL(c, EMB_ERR_ARG, "owner of table %d shard %d = %d not in [0, %d)", t, sh, o, c->G);
+      if ((sh == 0 && lo != 0) || lo < 0 || hi <= lo || hi > rows[t])
+        FAIL(c, EMB_ERR_ARG, "table %d shard %d rows [%lld, %lld) invalid", t, sh, (long long)lo, (long long)hi);
+      if (S == 1) {
+        c->owner[t] = o;
+        c->tables_of[o].push_back(t);
+      }
+      if (o == c->rank) {
+        lsh.push_back({t, sh, S > 1 ? ksh * c->S_max + sh : -1, lo, hi});
+        c->local.push_back(t);
+      }
+    }
+    if (S > 1) ++ksh;
   }
+  c->has_shard = c->T_sh > 0;
   c->T_r = (int)c->local.size();
   // contiguous batch split (C8)
   c->bstart.assign(c->G + 1, 0);
@@ -264,14 +306,21 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
     if (!w) FAIL(c, EMB_ERR_ARG, "local_weights[%d] is NULL", i);
     if (((uintptr_t)w) % 16 != 0) FAIL(c, EMB_ERR_ARG, "local_weights[%d] not 16-byte aligned", i);
     td[i].w = w;
-    td[i].rows = rows[c->local[i]];
-    td[i].tglob = c->local[i];
-    td[i].pad = 0;
+    td[i].rows = lsh[i].hi - lsh[i].lo;
+    td[i].tglob = lsh[i].t;
+    td[i].part = lsh[i].part;
+    td[i].lo = lsh[i].lo;
+  }
+  if (c->has_shard) {
+    CK(c, cudaMalloc(&c->d_comb_tglob, c->T_sh * sizeof(int32_t)));
+    CK(c, cudaMalloc(&c->d_comb_nsh, c->T_sh * sizeof(int32_t)));
+    CK(c, cudaMemcpy(c->d_comb_tglob, comb_tglob.data(), c->T_sh * sizeof(int32_t), cudaMemcpyHostToDevice));
+    CK(c, cudaMemcpy(c->d_comb_nsh, comb_nsh.data(), c->T_sh * sizeof(int32_t), cudaMemcpyHostToDevice));
   }
   CK(c, cudaMalloc(&c->d_tables, td.size() * sizeof(TableDesc)));
   CK(c, cudaMemcpy(c->d_tables, td.data(), td.size() * sizeof(TableDesc), cudaMemcpyHostToDevice));
   // unpack maps: recv = [G][B_r][T_src][d]; vector index of (b, t) = R0[src] + b*T_src + t_l
-  {
+  if (!c->has_shard) {
     const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
     std::vector<int64_t> base(num_tables);
     std::vector<int32_t> stride(num_tables);
@@ -295,6 +344,13 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   c->slot_off = 512;
   c->slot_bytes = round_up((size_t)Br * (size_t)num_tables * (size_t)dim * osz, 512);
   c->sym_bytes = c->slot_off + 2 * c->slot_bytes;
+  if (c->has_shard) {  // f3 partial slots [2][B_r][T_sh * S_max][d] fp32
+    if (dim % 4 != 0) FAIL(c, EMB_ERR_ARG, "row-sharded tables need dim %% 4 == 0");
+    c->part_off = c->sym_bytes;
+    c->pslot_bytes = round_up((size_t)Br * (size_t)c->T_sh * (size_t)c->S_max * (size_t)dim * 4, 512);
+    c->sym_bytes += 2 * c->pslot_bytes;
+  }
+  if (c->bwd_enabled && c->has_shard) FAIL(c, EMB_ERR_ARG, "backward with row-sharded tables is not supported");
   if (c->bwd_enabled) {
     if (!choose_tiling((int64_t)dim * 4, 4, 4, &c->blanes, &c->bvb, &c->bnv) || c->bnv > 4)
       FAIL(c, EMB_ERR_ARG, "backward: unsupported fp32 row size %d bytes", dim * 4);
@@ -320,6 +376,8 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   mine.slot_bytes = c->slot_bytes;
   mine.grad_off = c->grad_off;
   mine.gslot_bytes = c->gslot_bytes;
+  mine.part_off = c->part_off;
+  mine.pslot_bytes = c->pslot_bytes;
   mine.device = c->dev;
   CK(c, cudaIpcGetMemHandle(&mine.handle, c->sym));
   std::vector<PeerBlob> all(c->G);
@@ -334,6 +392,8 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
   c->peer_ipc.assign(c->G, false);
   c->peer_grad_off.assign(c->G, 0);
   c->peer_gslot_bytes.assign(c->G, 0);
+  c->peer_part_off.assign(c->G, 0);
+  c->peer_pslot_bytes.assign(c->G, 0);
   for (int p = 0; p < c->G; ++p) {
     const PeerBlob& b = all[p];
     if (b.magic != kMagic || b.rank != p) FAIL(c, EMB_ERR_PEER, "bad peer blob from rank %d", p);
@@ -342,6 +402,8 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
     c->peer_slot_bytes[p] = b.slot_bytes;
     c->peer_grad_off[p] = b.grad_off;
     c->peer_gslot_bytes[p] = b.gslot_bytes;
+    c->peer_part_off[p] = b.part_off;
+    c->peer_pslot_bytes[p] = b.pslot_bytes;
     if ((b.grad_off != 0) != c->bwd_enabled) FAIL(c, EMB_ERR_PEER, "rank %d disagrees on enable_backward", p);
     if (p == c->rank) {
       c->peer_base[p] = c->sym;
@@ -367,6 +429,70 @@ emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t
     if (c->ag(c->user, &one, r.data(), sizeof(int)) != 0) FAIL(c, EMB_ERR_PEER, "registration barrier failed");
   }
   c->registered = true;
+  // Load every kernel this context may launch now (CUDA lazy loading would otherwise load
+  // a kernel at its first launch, and a module load can wait for a running kernel -- e.g.
+  // the in-kernel peer wait of another rank sharing this GPU).
+  {
+    cudaFuncAttributes a;
+    const bool full = full_row(c);
+    for (int chk = 0; chk < 2; ++chk) {
+      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
+                                            full, c->sidx != 0, c->has_shard && chk == 0));
+      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
+                                            full, c->sidx != 0, false));
+    }
+    cudaFuncGetAttributes(&a, emb_wait_kernel);
+    cudaFuncGetAttributes(&a, emb_unpack_kernel);
+    cudaFuncGetAttributes(&a, emb_unpack8_kernel);
+    cudaFuncGetAttributes(&a, emb_combine_kernel<float>);
+    cudaFuncGetAttributes(&a, emb_combine_kernel<__nv_bfloat16>);
+    cudaFuncGetAttributes(&a, emb_bwd_signal_kernel);
+    cudaFuncGetAttributes(&a, emb_bwd_slot_wait_kernel);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4>);
+    cudaGetLastError();
+  }
+  return EMB_OK;
+}
+
+emb_status_t emb_register_tables(emb_ctx_t* c, int32_t num_tables, const int64_t* rows, const int32_t* owner,
+                                 int32_t dim, emb_dtype_t weight_dtype, emb_dtype_t out_dtype, int64_t global_batch,
+                                 const void* const* local_weights) {
+  if (!c) return EMB_ERR_ARG;
+  if (num_tables < 1 || !rows || !owner) FAIL(c, EMB_ERR_ARG, "num_tables/rows/owner invalid");
+  std::vector<int32_t> ns(num_tables, 1);
+  std::vector<int64_t> lo(num_tables, 0);
+  return register_impl(c, num_tables, rows, ns.data(), owner, lo.data(), dim, weight_dtype, out_dtype, global_batch,
+                       local_weights);
+}
+
+emb_status_t emb_register_sharded_tables(emb_ctx_t* c, int32_t num_tables, const int64_t* rows,
+                                         const int32_t* num_shards, const int32_t* shard_owner,
+                                         const int64_t* shard_row_start, int32_t dim, emb_dtype_t weight_dtype,
+                                         emb_dtype_t out_dtype, int64_t global_batch,
+                                         const void* const* local_weights) {
+  return register_impl(c, num_tables, rows, num_shards, shard_owner, shard_row_start, dim, weight_dtype, out_dtype,
+                       global_batch, local_weights);
+}
+
+static emb_status_t launch_combine(emb_ctx_t* c, cudaStream_t s) {
+  if (!c->has_shard) return EMB_OK;
+  const int slot = (int)(c->epoch & 1);
+  const float* part = reinterpret_cast<const float*>(c->sym + c->part_off + (size_t)slot * c->pslot_bytes);
+  char* out = c->sym + c->slot_off + (size_t)slot * c->slot_bytes;
+  const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  const int64_t total = Br * c->T_sh * (c->d / 4);
+  int grid = (int)std::min<int64_t>((total + kBlock - 1) / kBlock, (int64_t)c->num_sms * 8);
+  if (grid < 1) return EMB_OK;
+  if (c->odt == EMB_F32)
+    emb_combine_kernel<float><<<grid, kBlock, 0, s>>>(part, out, c->d_comb_tglob, c->d_comb_nsh, Br, c->T, c->T_sh,
+                                                      c->S_max, c->d);
+  else
+    emb_combine_kernel<__nv_bfloat16><<<grid, kBlock, 0, s>>>(part, out, c->d_comb_tglob, c->d_comb_nsh, Br, c->T,
+                                                              c->T_sh, c->S_max, c->d);
+  CK(c, cudaGetLastError());
   return EMB_OK;
 }
 
@@ -398,7 +524,10 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
     for (int g = 0; g < c->G; ++g) {
       p->out_base[g] = c->peer_base[g] + c->peer_slot_off[g] + (size_t)slot * c->peer_slot_bytes[g];
       p->peer_flag[g] = (g == c->rank) ? nullptr : reinterpret_cast<uint32_t*>(c->peer_base[g]) + c->rank;
+      if (c->has_shard)
+        p->part_base[g] = c->peer_base[g] + c->peer_part_off[g] + (size_t)slot * c->peer_pslot_bytes[g];
     }
+    p->part_stride = (int64_t)c->T_sh * c->S_max;
   } else {
     p->rowstride = c->T_r;
     p->use_tglob = 0;
@@ -413,7 +542,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 }
 
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0);
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0, p.part_stride > 0);
   const size_t smem = dyn_smem(c);
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
@@ -436,6 +565,8 @@ emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* in
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward before emb_register_tables");
   if (c->T_r > 0 && (!offsets || !indices)) FAIL(c, EMB_ERR_ARG, "offsets/indices NULL");
   CK(c, cudaSetDevice(c->dev));
+  if (c->has_shard && (flags & EMB_FWD_CHECK_BOUNDS))
+    FAIL(c, EMB_ERR_ARG, "EMB_FWD_CHECK_BOUNDS is not supported with row-sharded tables");
   c->epoch += 1;
   FwdParams p;
   fill_params(c, offsets, indices, true, nullptr, &p);
@@ -443,6 +574,10 @@ emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* in
   c->last = p;
   emb_status_t st = launch_fwd(c, p, flags, (cudaStream_t)stream);
   if (st != EMB_OK) return st;
+  if (!(flags & EMB_FWD_SEPARATE_WAIT)) {  // f3: partials landed (in-kernel wait) -> combine
+    st = launch_combine(c, (cudaStream_t)stream);
+    if (st != EMB_OK) return st;
+  }
   if (out) *out = c->sym + c->slot_off + (size_t)(c->epoch & 1) * c->slot_bytes;
   return EMB_OK;
 }
@@ -451,10 +586,11 @@ emb_status_t emb_wait(emb_ctx_t* c, void* stream) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered || c->epoch == 0) FAIL(c, EMB_ERR_STATE, "emb_wait without a forward");
   CK(c, cudaSetDevice(c->dev));
-  if (c->G == 1) return EMB_OK;
-  emb_wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(c->last);
-  CK(c, cudaGetLastError());
-  return EMB_OK;
+  if (c->G > 1) {
+    emb_wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(c->last);
+    CK(c, cudaGetLastError());
+  }
+  return launch_combine(c, (cudaStream_t)stream);
 }
 
 emb_status_t emb_forward_host(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
@@ -681,6 +817,8 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->d_tables) cudaFree(c->d_tables);
   if (c->ctrl) cudaFree(c->ctrl);
   if (c->d_unpack_base) cudaFree(c->d_unpack_base);
+  if (c->d_comb_tglob) cudaFree(c->d_comb_tglob);
+  if (c->d_comb_nsh) cudaFree(c->d_comb_nsh);
   if (c->d_unpack_stride) cudaFree(c->d_unpack_stride);
   if (c->d_off_stage) cudaFree(c->d_off_stage);
   if (c->d_idx_stage) cudaFree(c->d_idx_stage);
@@ -795,6 +933,7 @@ const char* emb_last_error(const emb_ctx_t* c) { return c ? c->err.c_str() : g_i
 emb_status_t emb_baseline_splits(const emb_ctx_t* c, int64_t* send_counts, int64_t* recv_counts) {
   if (!c || !send_counts || !recv_counts) return EMB_ERR_ARG;
   if (!c->registered) return EMB_ERR_STATE;
+  if (c->has_shard) return EMB_ERR_ARG;
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   for (int g = 0; g < c->G; ++g) {
     send_counts[g] = (c->bstart[g + 1] - c->bstart[g]) * c->T_r * c->d;
@@ -807,6 +946,7 @@ emb_status_t emb_baseline_pool(emb_ctx_t* c, const int64_t* offsets, const int64
                                void* stream, void* send) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_pool before emb_register_tables");
+  if (c->has_shard) FAIL(c, EMB_ERR_ARG, "the comparison path does not support row-sharded tables");
   if (c->T_r > 0 && (!offsets || !indices || !send)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
   CK(c, cudaSetDevice(c->dev));
   FwdParams p;
@@ -817,6 +957,7 @@ emb_status_t emb_baseline_pool(emb_ctx_t* c, const int64_t* offsets, const int64
 emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, void* out) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_unpack before emb_register_tables");
+  if (c->has_shard) FAIL(c, EMB_ERR_ARG, "the comparison path does not support row-sharded tables");
   if (!recv || !out) FAIL(c, EMB_ERR_ARG, "NULL buffer");
   CK(c, cudaSetDevice(c->dev));
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];

@@ -111,6 +111,22 @@ def emb_register_tables(ctx: EmbCtx, rows: Sequence[int], owner: Sequence[int], 
     _check(ctx, st)
 
 
+def emb_register_sharded_tables(ctx: EmbCtx, rows: Sequence[int], num_shards: Sequence[int],
+                                shard_owner: Sequence[int], shard_row_start: Sequence[int], dim: int, weight_dtype,
+                                out_dtype, global_batch: int, local_weights: Sequence) -> None:
+    T = len(rows)
+    n = sum(int(x) for x in num_shards)
+    rows_a = (C.c_int64 * T)(*[int(r) for r in rows])
+    ns_a = (C.c_int32 * T)(*[int(x) for x in num_shards])
+    own_a = (C.c_int32 * n)(*[int(o) for o in shard_owner])
+    lo_a = (C.c_int64 * n)(*[int(x) for x in shard_row_start])
+    nl = len(local_weights)
+    w_a = (C.c_void_p * max(nl, 1))(*[_ptr(w) for w in local_weights])
+    st = _lib.lib().emb_register_sharded_tables(ctx, T, rows_a, ns_a, own_a, lo_a, int(dim), _dtype_code(weight_dtype),
+                                                _dtype_code(out_dtype), int(global_batch), w_a)
+    _check(ctx, st)
+
+
 def emb_forward(ctx: EmbCtx, offsets, indices, flags: int = 0, stream=None) -> int:
     """Returns the device address of this epoch's Y_r = [B_r][T][d]."""
     out = C.c_void_p()

@@ -37,13 +37,19 @@ class PgasEmbedding:
 
     def __init__(self, rank: int, world_size: int, device: int, rows: Sequence[int], owner: Sequence[int], dim: int,
                  local_weights: Sequence[torch.Tensor], global_batch: int, weight_dtype="f32", out_dtype="f32",
-                 allgather=None, options: Optional[dict] = None, backward: bool = False):
+                 allgather=None, options: Optional[dict] = None, backward: bool = False, shards=None):
         self.device = torch.device("cuda", device)
         self.ctx = E.emb_init(rank, world_size, device, allgather)
         if backward:
             E.emb_set_option(self.ctx, "enable_backward", 1)
         self._weights = list(local_weights)  # zero-copy: keep alive
-        E.emb_register_tables(self.ctx, rows, owner, dim, weight_dtype, out_dtype, global_batch, self._weights)
+        if shards is None:
+            E.emb_register_tables(self.ctx, rows, owner, dim, weight_dtype, out_dtype, global_batch, self._weights)
+        else:  # f3: shards = [(t, s, lo, hi, owner)], local_weights in ascending (t, s) of this rank
+            sh = sorted((int(t), int(s_), int(lo), int(o)) for (t, s_, lo, hi, o) in shards)
+            nsh = [sum(1 for x in sh if x[0] == t) for t in range(len(rows))]
+            E.emb_register_sharded_tables(self.ctx, rows, nsh, [x[3] for x in sh], [x[2] for x in sh], dim,
+                                          weight_dtype, out_dtype, global_batch, self._weights)
         for k, v in (options or {}).items():
             E.emb_set_option(self.ctx, k, v)
         self.info = E.emb_get_info(self.ctx)
