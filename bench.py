@@ -49,6 +49,9 @@ def parse():
     p.add_argument("--no-control", action="store_true", help="skip the uniform-index control measurement")
     p.add_argument("--no-compare", action="store_true", help="skip the NCCL comparison path")
     p.add_argument("--opt", action="append", default=[], help="libemb option key=value")
+    p.add_argument("--shards", type=int, default=1,
+                   help="f3: split every table into this many row shards (owners round-robin from the table's owner);"
+                        " the kernel partitions the full CSR in-kernel and combines partials in shard order")
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                    help="process-group backend (gloo: test harness only; a2a staged through host)")
     p.add_argument("--same-device", action="store_true",
@@ -70,7 +73,8 @@ def config_desc(w, N):
             "pooling": f"U{{{w.pmin}..{w.pmax}}}", "indices": f"{w.dist}({w.alpha})" if w.dist == "zipf" else "uniform",
             "weights": w.wdtype, "out": w.odtype, "parallelism": f"table-wise MP x{N} + batch DP x{N}",
             "aliased": int(w.T // (int(w.phys.max()) + 1)) if int(w.phys.max()) + 1 < w.T else 1,
-            "l2": "inputs larger than L2 (tables >> 126 MB, rotating CSR batches); no flush"}
+            "l2": "inputs larger than L2 (tables >> 126 MB, rotating CSR batches); no flush",
+            "row_shards_per_table": getattr(w, "_shards", 1)}
 
 
 def unique_rows(w, rank, batch):
@@ -327,10 +331,42 @@ def main():
     for kv in args.opt:
         k, v = kv.split("=")
         opts[k] = int(v)
-    layer = PgasEmbedding(rank, N, local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
-                          torch_allgather() if N > 1 else None, opts, backward=(args.mode == "backward"))
     nnz = [int(b[0][-1].item()) for b in batches]
     uniq = [unique_rows(w, rank, b) for b in batches]     # untimed: compulsory-traffic basis
+    w._shards = args.shards
+    shards = None
+    if args.shards > 1:
+        # f3: table t -> S row shards, shard s on rank (owner[t] + s) % N; each rank needs the
+        # FULL CSR of every table it holds a shard of.  Tables are generated where the
+        # table's owner is; at N = 1 every shard is a view of the local table.
+        if N > 1:
+            raise SystemExit("--shards > 1 is exercised at N = 1 in this round (all shards local)")
+        args.no_control = True       # the uniform control and the comparison path are table-wise
+        args.no_compare = True
+        S = args.shards
+        shards = []
+        for t in range(w.T):
+            cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(np.int64)
+            for sh in range(S):
+                shards.append((t, sh, int(cuts[sh]), int(cuts[sh + 1]), (int(w.owner[t]) + sh) % N))
+        tables = [tables[list(w.local_tables(rank)).index(t)][lo:hi] for (t, sh, lo, hi, o) in sorted(shards)]
+
+        def shard_csr(batch):
+            off, idx = batch
+            lt = list(w.local_tables(rank))
+            o_parts, x_parts, base = [torch.zeros(1, dtype=torch.int64, device=dev)], [], 0
+            for (t, sh, lo, hi, o) in sorted(shards):
+                tl = lt.index(t)
+                seg = off[tl * w.B: (tl + 1) * w.B + 1]
+                o_parts.append(seg[1:] - seg[0] + base)
+                x_parts.append(idx[int(seg[0]): int(seg[-1])])
+                base += int(seg[-1] - seg[0])
+            return torch.cat(o_parts), torch.cat(x_parts)
+        batches = [shard_csr(b) for b in batches]
+        torch.cuda.synchronize()
+    layer = PgasEmbedding(rank, N, local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
+                          torch_allgather() if N > 1 else None, opts, backward=(args.mode == "backward"),
+                          shards=shards)
     T_r = len(w.local_tables(rank))
     nbags = T_r * w.B
     B_r = layer.B_r
