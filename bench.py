@@ -161,7 +161,7 @@ class OracleSampler:
     this rank's tables over the full batch plus the MP->DP layout step; extrapolate
     to the whole rank workload by table count.  Inputs are generated once, untimed."""
 
-    def __init__(self, w, rank, max_tables=8):
+    def __init__(self, w, rank, max_tables=64):
         from oracle import emb_oracle as O
         self.O = O
         self.w = w
@@ -194,7 +194,7 @@ class OracleSampler:
                 "seconds": dt, "rank_seconds": per_rank_s}
 
 
-def oracle_sample(w, rank, budget_s=12.0):
+def oracle_sample(w, rank, budget_s=20.0):
     return OracleSampler(w, rank).run(budget_s)
 
 
