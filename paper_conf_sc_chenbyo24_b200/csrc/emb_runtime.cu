@@ -547,7 +547,9 @@ static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags,
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
   // carve-out that fits (the rest of the 256 KB per SM becomes L1)
-  if (c->carveout >= 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, c->carveout));
+  // (only without dynamic shared memory: a 0 % carve-out would cap residency at 1 CTA/SM)
+  if (c->carveout >= 0 && smem == 0)
+    CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, c->carveout));
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0) {
     CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem));
