@@ -35,6 +35,7 @@ struct BwdParams {
   Ctrl* ctrl;                  // uses bwork / bdone
   int64_t timeout_ns;
   int32_t T, T_r, d, G, rank, lanes, chunk_rows;
+  int32_t interleave;          // 1: chunk c -> table c mod T_r (spreads same-row atomics over time)
   uint32_t epoch;
 };
 
@@ -106,8 +107,10 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
       if (lane == 0) c = atomicAdd(&p.ctrl->bwork, 1u);
       c = __shfl_sync(kFull, c, 0);
       if ((int64_t)c >= nchunks) break;
-      const int t_l = (int)(c / cpt);
-      const int64_t b0 = ((int64_t)c % cpt) * cb;
+      // interleave tables (chunk c -> table c mod T_r): a zipf-hot dW row then receives its
+      // atomics spread over the whole kernel instead of from every warp at once
+      const int t_l = p.interleave ? (int)(c % p.T_r) : (int)(c / cpt);
+      const int64_t b0 = (p.interleave ? (int64_t)(c / p.T_r) : (int64_t)c % cpt) * cb;
       const int nb = (int)min((int64_t)cb, B - b0);
       const int64_t o_l = (lane <= nb) ? ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane) : 0;
       const TableDesc* tdp = p.tables + t_l;

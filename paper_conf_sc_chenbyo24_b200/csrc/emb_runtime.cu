@@ -118,6 +118,7 @@ struct emb_ctx {
   std::vector<uint64_t> peer_grad_off, peer_gslot_bytes;
   uint64_t bepoch = 0;
   bool bwd_ready_pending = false;
+  int bwd_interleave = 1;
   float** d_dW = nullptr;
   std::vector<void*> h_dW;
   int blanes = 32, bvb = 16, bnv = 1;
@@ -718,6 +719,7 @@ static void fill_bwd_params(emb_ctx_t* c, BwdParams* p) {
   p->rank = c->rank;
   p->lanes = c->blanes;
   p->chunk_rows = c->chunk_rows;
+  p->interleave = c->bwd_interleave;
   p->epoch = (uint32_t)c->bepoch;
 }
 
@@ -897,6 +899,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->minblocks = (int)v;
   }
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
+  else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "carveout")) {
     if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");
     c->carveout = (int)v;
