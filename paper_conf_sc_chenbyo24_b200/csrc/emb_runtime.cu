@@ -119,6 +119,7 @@ struct emb_ctx {
   uint64_t bepoch = 0;
   bool bwd_ready_pending = false;
   int bwd_interleave = 1;
+  int fwd_interleave = 0;
   float** d_dW = nullptr;
   std::vector<void*> h_dW;
   int blanes = 32, bvb = 16, bnv = 1;
@@ -511,6 +512,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   p->lanes = c->lanes;
   p->chunk_rows = c->chunk_rows;
   p->stagger = c->stagger;
+  p->interleave = c->fwd_interleave;
   p->ctrl = c->ctrl;
   p->timeout_ns = c->timeout_ns;
   for (int g = 0; g <= c->G; ++g) p->bstart[g] = c->bstart[g];
@@ -900,6 +902,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   }
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
+  else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "carveout")) {
     if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");
     c->carveout = (int)v;

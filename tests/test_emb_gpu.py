@@ -336,7 +336,7 @@ VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),
 @pytest.mark.parametrize("opts", [{"unroll": 2}, {"unroll": 4}, {"unroll": 8}, {"unroll": 16},
                                   {"unroll": 4, "minblocks": 1}, {"unroll": 4, "minblocks": 6},
                                   {"chunk_rows": 1}, {"chunk_rows": 100000}, {"stagger": 0}, {"sidx": 1},
-                                  {"sidx": 1, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}])
+                                  {"sidx": 1, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}, {"fwd_interleave": 1}])
 @pytest.mark.parametrize("case", range(len(VARIANT_CASES)))
 def test_pipeline_variants_bitexact(opts, case):
     """Every register/shared-memory pipeline variant and chunking is bit-exact."""
