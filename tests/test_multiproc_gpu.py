@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _worker(rank, G, port, q, flags, owner, epochs):
+def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -51,7 +51,12 @@ def _worker(rank, G, port, q, flags, owner, epochs):
         for ep in range(epochs):
             o, x = synth.rank_csr(w, 500 + ep, rank)
             ref = H.oracle_outputs(w, 500 + ep, tabs)[rank]
-            y = layer.forward(torch.from_numpy(o).to(dev), torch.from_numpy(x).to(dev), flags, s)
+            od, xd = torch.from_numpy(o).to(dev), torch.from_numpy(x).to(dev)
+            if rank == delay_rank:                    # fault injection: this rank arrives late
+                import time
+                time.sleep(0.3)
+                torch.cuda._sleep(50_000_000)         # ~25 ms of GPU spin ahead of its forward
+            y = layer.forward(od, xd, flags, s)
             if flags & E.EMB_FWD_SEPARATE_WAIT:
                 layer.wait(s)
             s.synchronize()
@@ -69,13 +74,14 @@ def _worker(rank, G, port, q, flags, owner, epochs):
         q.put((rank, False, -1, traceback.format_exc()))
 
 
-@pytest.mark.parametrize("G,flags,owner", [(2, 0, None), (3, 0, [2, 2, 0, 1, 0, 2]), (2, 2, None)])
-def test_cross_process_ipc_pgas(G, flags, owner):
+@pytest.mark.parametrize("G,flags,owner,delay", [(2, 0, None, -1), (3, 0, [2, 2, 0, 1, 0, 2], -1), (2, 2, None, -1),
+                                                (3, 0, None, 1), (2, 2, None, 0)])
+def test_cross_process_ipc_pgas(G, flags, owner, delay):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    ps = [ctx.Process(target=_worker, args=(r, G, port, q, flags, owner, 4)) for r in range(G)]
+    ps = [ctx.Process(target=_worker, args=(r, G, port, q, flags, owner, 4, delay)) for r in range(G)]
     for p in ps:
         p.start()
     res = []
