@@ -30,6 +30,9 @@
  *   - Device pointers are plain CUDA device addresses of the context's device.
  *   - Collective calls (emb_register_tables, emb_forward, emb_finalize) must be
  *     entered by every rank, in the same order.
+ *   - One forward-type launch (emb_forward / emb_baseline_pool) in flight per context at a
+ *     time: they share the context's device work counters (stream order provides this when
+ *     they are issued on one stream).
  *   - Readings of points the paper leaves open are listed in DESIGN.md (C1..C29).
  */
 #ifndef EMB_H_
