@@ -4,8 +4,8 @@
 
 namespace emb {
 using KernelFn = void (*)(FwdParams);
-KernelFn pick_tile_f32_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard);
-KernelFn pick_tile_f32_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard);
-KernelFn pick_tile_bf16_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard);
-KernelFn pick_tile_bf16_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard);
+KernelFn pick_tile_f32_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast);
+KernelFn pick_tile_f32_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast);
+KernelFn pick_tile_bf16_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast);
+KernelFn pick_tile_bf16_bf16(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast);
 }  // namespace emb

@@ -4,7 +4,13 @@
 namespace emb {
 namespace {
 template <int VB, int NV, typename WT, typename OT, bool CHECK>
-KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard) {
+KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard, bool tmast) {
+  if constexpr (!CHECK && NV == 1) {
+    if (tmast && full && !shard) {  // f4: staged vectors shipped by TMA scatter4
+      if (unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, false, 6, true, false, false, true>;
+      return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, false, false, true>;
+    }
+  }
   if constexpr (!CHECK) {
     if (shard) {  // f3: row-sharded tables (in-kernel id partitioning, partial slots)
       if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, false, false, true>;
@@ -26,8 +32,8 @@ KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard) {
   }
 }
 template <int VB, int NV, typename WT, typename OT>
-KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx, bool shard) {
-  if (unroll >= 8 && !shard) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
+KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast) {
+  if (unroll >= 8 && !shard && !tmast) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
     if constexpr (NV == 1) {
       if (unroll == 16)
         return check ? emb_fwd_async_kernel<VB, NV, WT, OT, 16, true, 3> : emb_fwd_async_kernel<VB, NV, WT, OT, 16, false, 3>;
@@ -35,20 +41,20 @@ KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx, bool shard
     }
     unroll = 4;
   }
-  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full, sidx, shard)
-               : pick_u<VB, NV, WT, OT, false>(unroll, mb, full, sidx, shard);
+  return check ? pick_u<VB, NV, WT, OT, true>(unroll, mb, full, sidx, shard, tmast)
+               : pick_u<VB, NV, WT, OT, false>(unroll, mb, full, sidx, shard, tmast);
 }
 }  // namespace
 
-KernelFn pick_tile_bf16_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard) {
+KernelFn pick_tile_bf16_f32(int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast) {
   using WT = __nv_bfloat16;
   using OT = float;
-  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full, sidx, shard);
+  if (vb == 8) return pick_c<8, 1, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
   switch (nv) {
-    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full, sidx, shard);
-    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full, sidx, shard);
-    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full, sidx, shard);
-    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx, shard);
+    case 2: return pick_c<16, 2, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
+    case 4: return pick_c<16, 4, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
+    case 8: return pick_c<16, 8, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
+    default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
   }
 }
 }  // namespace emb

@@ -7,6 +7,8 @@
 // symmetric `outputs` array addressed on any PE (L216, L228, L232) becomes a
 // cudaMalloc'd buffer per rank whose IPC handle is all-gathered once over the
 // caller's process group.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <unistd.h>
 
@@ -120,6 +122,8 @@ struct emb_ctx {
   bool bwd_ready_pending = false;
   int bwd_interleave = 1;
   int fwd_interleave = 0;
+  int tma_store = 0;          // f4: stage pooled vectors, ship 4 per TMA scatter4
+  void* d_tmaps = nullptr;    // f4: CUtensorMap [2 slots][kMaxG] of every rank's output slots
   float** d_dW = nullptr;
   std::vector<void*> h_dW;
   int blanes = 32, bvb = 16, bnv = 1;
@@ -163,11 +167,11 @@ static size_t dyn_smem(const emb_ctx* c) {
 // ---------------------------------------------------------------------------- kernel dispatch
 namespace {
 
-KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard = false) {
-  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx, shard);
-  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx, shard);
-  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx, shard);
-  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx, shard);
+KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard = false, bool tmast = false) {
+  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
+  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
+  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
+  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
 }
 
 // row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
@@ -498,6 +502,39 @@ static emb_status_t launch_combine(emb_ctx_t* c, cudaStream_t s) {
   return EMB_OK;
 }
 
+// f4: one 2-D tensor map per (slot, destination rank) over that rank's output slot viewed
+// as [B_dst*T rows][d], box = one row; the kernel scatters 4 rows per TMA store
+static emb_status_t build_tmaps(emb_ctx_t* c) {
+  if (c->d_tmaps) return EMB_OK;
+  if (!full_row(c) || c->nv != 1 || c->has_shard || c->d > 256)
+    FAIL(c, EMB_ERR_ARG, "tma_store needs full-warp rows with one vector per lane, d <= 256, no row sharding");
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  CK(c, cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+  if (!fn || q != cudaDriverEntryPointSuccess) FAIL(c, EMB_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  std::vector<CUtensorMap> maps(2 * kMaxG);
+  memset(maps.data(), 0, maps.size() * sizeof(CUtensorMap));
+  const size_t eo = esize(c->odt);
+  for (int slot = 0; slot < 2; ++slot)
+    for (int g = 0; g < c->G; ++g) {
+      void* base = c->peer_base[g] + c->peer_slot_off[g] + (size_t)slot * c->peer_slot_bytes[g];
+      const cuuint64_t rows = (cuuint64_t)(c->bstart[g + 1] - c->bstart[g]) * (cuuint64_t)c->T;
+      cuuint64_t dims[2] = {(cuuint64_t)c->d, rows};
+      cuuint64_t strides[1] = {(cuuint64_t)c->d * eo};
+      cuuint32_t box[2] = {(cuuint32_t)c->d, 1};
+      cuuint32_t es[2] = {1, 1};
+      CUresult r = encode(&maps[slot * kMaxG + g],
+                          c->odt == EMB_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                          base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) FAIL(c, EMB_ERR_CUDA, "cuTensorMapEncodeTiled(slot %d, rank %d) failed: %d", slot, g, (int)r);
+    }
+  CK(c, cudaMalloc(&c->d_tmaps, maps.size() * sizeof(CUtensorMap)));
+  CK(c, cudaMemcpy(c->d_tmaps, maps.data(), maps.size() * sizeof(CUtensorMap), cudaMemcpyHostToDevice));
+  return EMB_OK;
+}
+
 static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, bool pgas, char* send,
                                 FwdParams* p) {
   memset(p, 0, sizeof(*p));
@@ -531,6 +568,8 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
         p->part_base[g] = c->peer_base[g] + c->peer_part_off[g] + (size_t)slot * c->peer_pslot_bytes[g];
     }
     p->part_stride = (int64_t)c->T_sh * c->S_max;
+    p->tmaps = (c->tma_store && c->d_tmaps) ? static_cast<const char*>(c->d_tmaps) + (size_t)slot * kMaxG * sizeof(CUtensorMap)
+                                            : nullptr;
   } else {
     p->rowstride = c->T_r;
     p->use_tglob = 0;
@@ -545,8 +584,9 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 }
 
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0, p.part_stride > 0);
-  const size_t smem = dyn_smem(c);
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0, p.part_stride > 0, p.tmaps != nullptr);
+  size_t smem = dyn_smem(c);
+  if (p.tmaps) smem = std::max(smem, (size_t)(kBlock / 32) * 8 * c->d * esize(c->odt));  // f4 staging (2 x 4 rows)
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
   // carve-out that fits (the rest of the 256 KB per SM becomes L1)
@@ -572,6 +612,10 @@ emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* in
   CK(c, cudaSetDevice(c->dev));
   if (c->has_shard && (flags & EMB_FWD_CHECK_BOUNDS))
     FAIL(c, EMB_ERR_ARG, "EMB_FWD_CHECK_BOUNDS is not supported with row-sharded tables");
+  if (c->tma_store) {
+    emb_status_t st0 = build_tmaps(c);
+    if (st0 != EMB_OK) return st0;
+  }
   c->epoch += 1;
   FwdParams p;
   fill_params(c, offsets, indices, true, nullptr, &p);
@@ -824,6 +868,7 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->ctrl) cudaFree(c->ctrl);
   if (c->d_unpack_base) cudaFree(c->d_unpack_base);
   if (c->d_comb_tglob) cudaFree(c->d_comb_tglob);
+  if (c->d_tmaps) cudaFree(c->d_tmaps);
   if (c->d_comb_nsh) cudaFree(c->d_comb_nsh);
   if (c->d_unpack_stride) cudaFree(c->d_unpack_stride);
   if (c->d_off_stage) cudaFree(c->d_off_stage);
@@ -903,6 +948,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
+  else if (!strcmp(key, "tma_store")) c->tma_store = v ? 1 : 0;
   else if (!strcmp(key, "carveout")) {
     if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");
     c->carveout = (int)v;
