@@ -33,6 +33,17 @@ KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard, bool tmast
 }
 template <int VB, int NV, typename WT, typename OT>
 KernelFn pick_c(int unroll, bool check, int mb, bool full, bool sidx, bool shard, bool tmast) {
+  if constexpr (NV == 1) {  // ring v2: cp.async rows, more rows in flight than registers allow
+    if (!check && full && !shard && !tmast && unroll < 0) {
+      switch (-unroll) {
+        case 8: return emb_fwd_ring_kernel<VB, WT, OT, 8, 6>;
+        case 12: return emb_fwd_ring_kernel<VB, WT, OT, 12, 4>;
+        case 16: return emb_fwd_ring_kernel<VB, WT, OT, 16, 3>;
+        default: return emb_fwd_ring_kernel<VB, WT, OT, 8, 4>;
+      }
+    }
+  }
+  if (unroll < 0) unroll = 4;
   if (unroll >= 8 && !shard && !tmast) {  // shared-memory ring (cp.async) with `unroll` rows in flight per warp
     if constexpr (NV == 1) {
       if (unroll == 16)

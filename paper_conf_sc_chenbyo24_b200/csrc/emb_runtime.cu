@@ -159,6 +159,8 @@ static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb 
 static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
 static size_t dyn_smem(const emb_ctx* c) {
+  if (eff_unroll(c) < 0 && c->nv == 1 && full_row(c) && !c->has_shard)  // ring v2: R rows of 512 B per warp
+    return (size_t)(kBlock / 32) * (size_t)(-eff_unroll(c) == 4 ? 8 : -eff_unroll(c)) * 32 * c->vb;
   if (eff_unroll(c) >= 8 && c->nv == 1) return (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb;
   if (c->sidx && c->nv == 1 && full_row(c)) return (size_t)(kBlock / 32) * 1024;  // id ring: 4 x 32 x 8 B per warp
   return 0;
@@ -938,7 +940,8 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "stagger")) c->stagger = v ? 1 : 0;
   else if (!strcmp(key, "timeout_ms")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "timeout_ms < 1"); c->timeout_ns = v * 1000000ll; }
   else if (!strcmp(key, "unroll")) {
-    if (v != 0 && v != 2 && v != 4 && v != 8 && v != 16) FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline) or 8, 16 (shared-memory ring)");
+    if (v != 0 && v != 2 && v != 4 && v != 8 && v != 16 && v != -4 && v != -8 && v != -12 && v != -16)
+      FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline), 8, 16 (cp.async ring) or -4/-8/-12/-16 (ring v2)");
     c->unroll = (int)v;
   }
   else if (!strcmp(key, "minblocks")) {

@@ -337,13 +337,14 @@ VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),
                                   {"unroll": 4, "minblocks": 1}, {"unroll": 4, "minblocks": 6},
                                   {"chunk_rows": 1}, {"chunk_rows": 100000}, {"stagger": 0}, {"sidx": 1},
                                   {"sidx": 1, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}, {"fwd_interleave": 1},
-                                  {"tma_store": 1}, {"tma_store": 1, "chunk_rows": 3}])
+                                  {"tma_store": 1}, {"tma_store": 1, "chunk_rows": 3}, {"unroll": -8}, {"unroll": -16},
+                                  {"unroll": -12, "chunk_rows": 5}])
 @pytest.mark.parametrize("case", range(len(VARIANT_CASES)))
 def test_pipeline_variants_bitexact(opts, case):
     """Every register/shared-memory pipeline variant and chunking is bit-exact."""
     w = synth.make_workload("tiny", G=2, T=5, **VARIANT_CASES[case])
-    if opts.get("tma_store") and w.dim * w.elem_bytes() < 256:
-        pytest.skip("tma_store needs full-warp rows (256 B+)")
+    if (opts.get("tma_store") or opts.get("unroll", 0) < 0) and w.dim * w.elem_bytes() < 256:
+        pytest.skip("tma_store / ring v2 need full-warp rows (256 B+)")
     tabs = H.np_tables(w)
     csr = H.np_csrs(w, 71)
     ref = H.oracle_outputs(w, 71, tabs, csr)
