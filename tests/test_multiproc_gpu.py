@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1):
+def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1, opts=None):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -39,13 +39,14 @@ def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1):
 
         torch.cuda.set_device(0)
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=G)
-        w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=97, T=6, dim=32, rows=600,
+        dim = 64 if (opts or {}).get("tma_store") else 32   # TMA scatter4 needs rows >= 256 B
+        w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=97, T=6, dim=dim, rows=600,
                                 owner=np.array(owner) if owner else None)
         tabs = H.np_tables(w)
         dev = torch.device("cuda", 0)
         local = [torch.from_numpy(tabs[int(w.phys[t])]).to(dev) for t in w.local_tables(rank)]
         layer = PgasEmbedding(rank, G, 0, w.rows, w.owner, w.dim, local, w.B, "f32", "f32", torch_allgather(),
-                              {"timeout_ms": 20000})
+                              {"timeout_ms": 20000, **(opts or {})})
         ok = True
         s = torch.cuda.Stream()
         for ep in range(epochs):
@@ -74,14 +75,16 @@ def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1):
         q.put((rank, False, -1, traceback.format_exc()))
 
 
-@pytest.mark.parametrize("G,flags,owner,delay", [(2, 0, None, -1), (3, 0, [2, 2, 0, 1, 0, 2], -1), (2, 2, None, -1),
-                                                (3, 0, None, 1), (2, 2, None, 0)])
-def test_cross_process_ipc_pgas(G, flags, owner, delay):
+@pytest.mark.parametrize("G,flags,owner,delay,opts", [(2, 0, None, -1, None), (3, 0, [2, 2, 0, 1, 0, 2], -1, None),
+                                                     (2, 2, None, -1, None), (3, 0, None, 1, None), (2, 2, None, 0, None),
+                                                     (3, 0, None, -1, {"tma_store": 1}),
+                                                     (2, 0, None, -1, {"unroll": -8})])
+def test_cross_process_ipc_pgas(G, flags, owner, delay, opts):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    ps = [ctx.Process(target=_worker, args=(r, G, port, q, flags, owner, 4, delay)) for r in range(G)]
+    ps = [ctx.Process(target=_worker, args=(r, G, port, q, flags, owner, 4, delay, opts)) for r in range(G)]
     for p in ps:
         p.start()
     res = []
