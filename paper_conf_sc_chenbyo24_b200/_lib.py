@@ -7,6 +7,8 @@ import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libemb.so")
+if os.environ.get("EMB_LIB"):            # experiment builds (build.build_variant) only
+    LIB_PATH = os.environ["EMB_LIB"]
 
 EMB_OK, EMB_ERR_ARG, EMB_ERR_STATE, EMB_ERR_CUDA, EMB_ERR_NOMEM, EMB_ERR_PEER, EMB_ERR_TIMEOUT, EMB_ERR_BOUNDS = range(8)
 STATUS_NAMES = ["EMB_OK", "EMB_ERR_ARG", "EMB_ERR_STATE", "EMB_ERR_CUDA", "EMB_ERR_NOMEM", "EMB_ERR_PEER",

@@ -47,17 +47,32 @@ def _nvcc(args):
     return r.stderr
 
 
+def build_variant(tag: str, defines) -> str:
+    """Experiment build of libemb with extra -D flags into exp/libemb_<tag>.so (selected at
+    load time with EMB_LIB=<path>; the default library is untouched)."""
+    spec = dict(LIBS["emb"])
+    spec["out"] = os.path.join(PKG, "exp", f"libemb_{tag}.so")
+    os.makedirs(os.path.dirname(spec["out"]), exist_ok=True)
+    _build_one(f"emb_{tag}", spec, True, False, [f"-D{d}" for d in defines])
+    return spec["out"]
+
+
 def build(names=None, force: bool = False, verbose: bool = False) -> None:
     """Compile every translation unit to an object in parallel, then link the .so."""
-    from concurrent.futures import ThreadPoolExecutor
     for name, spec in LIBS.items():
         if names and name not in names:
             continue
+        _build_one(name, spec, force, verbose)
+
+
+def _build_one(name, spec, force, verbose, extra=()):
+    from concurrent.futures import ThreadPoolExecutor
+    if True:
         if not force and not _stale(spec):
-            continue
+            return
         objdir = os.path.join(os.path.dirname(spec["out"]), ".obj")
         os.makedirs(objdir, exist_ok=True)
-        comp = [f for f in FLAGS if f != "-shared"]
+        comp = [f for f in FLAGS if f != "-shared"] + list(extra)
         jobs = []
         for src in spec["srcs"]:
             obj = os.path.join(objdir, os.path.basename(src) + ".o")

@@ -95,7 +95,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 0, carveout = 0;  // 0: auto per tile
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 1, carveout = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -122,6 +122,7 @@ struct emb_ctx {
   bool bwd_ready_pending = false;
   int bwd_interleave = 1;
   int fwd_interleave = 0;
+  int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
   int tma_store = 0;          // f4: stage pooled vectors, ship 4 per TMA scatter4
   void* d_tmaps = nullptr;    // f4: CUtensorMap [2 slots][kMaxG] of every rank's output slots
   float** d_dW = nullptr;
@@ -157,12 +158,21 @@ static int eff_minblocks(const emb_ctx* c) { return c->minblocks ? c->minblocks 
 static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4); }
 // a row exactly covers the warp's 32 lane vectors (lets the row stride be a constant)
 static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
+// the SIDX id ring (4 x 32 32-bit ids per warp in shared memory, LDS.128 broadcast of 4 ids
+// per row group) is on by default where the kernel has it: full-row tiles with one vector
+// per lane, no bounds check, no row shards, direct stores, 4-row groups (or 2 with 8-B lanes)
+static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
+  const int u = c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4);
+  const int mb = c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1);
+  return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
+         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && mb == 4) || u == 2);
+}
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
-static size_t dyn_smem(const emb_ctx* c) {
+static size_t dyn_smem(const emb_ctx* c, bool sidx = false) {
   if (eff_unroll(c) < 0 && c->nv == 1 && full_row(c) && !c->has_shard)  // ring v2: R rows of 512 B per warp
     return (size_t)(kBlock / 32) * (size_t)(-eff_unroll(c) == 4 ? 8 : -eff_unroll(c)) * 32 * c->vb;
   if (eff_unroll(c) >= 8 && c->nv == 1) return (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb;
-  if (c->sidx && c->nv == 1 && full_row(c)) return (size_t)(kBlock / 32) * 1024;  // id ring: 4 x 32 x 8 B per warp
+  if (sidx) return (size_t)(kBlock / 32) * 512;   // id ring: 4 x 32 x 4 B per warp
   return 0;
 }
 
@@ -445,9 +455,12 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     const bool full = full_row(c);
     for (int chk = 0; chk < 2; ++chk) {
       cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
-                                            full, c->sidx != 0, c->has_shard && chk == 0));
+                                            full, sidx_on(c, chk != 0, c->has_shard && chk == 0, false),
+                                            c->has_shard && chk == 0));
       cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
-                                            full, c->sidx != 0, false));
+                                            full, sidx_on(c, chk != 0, false, false), false));
+      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
+                                            full, false, false));
     }
     cudaFuncGetAttributes(&a, emb_wait_kernel);
     cudaFuncGetAttributes(&a, emb_unpack_kernel);
@@ -552,6 +565,8 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   p->chunk_rows = c->chunk_rows;
   p->stagger = c->stagger;
   p->interleave = c->fwd_interleave;
+  p->row_l2 = c->row_l2;
+  p->out_l2 = c->out_l2;
   p->ctrl = c->ctrl;
   p->timeout_ns = c->timeout_ns;
   for (int g = 0; g <= c->G; ++g) p->bstart[g] = c->bstart[g];
@@ -586,8 +601,10 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 }
 
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), (flags & EMB_FWD_CHECK_BOUNDS) != 0, eff_minblocks(c), full_row(c), c->sidx != 0, p.part_stride > 0, p.tmaps != nullptr);
-  size_t smem = dyn_smem(c);
+  const bool chk = (flags & EMB_FWD_CHECK_BOUNDS) != 0, shard = p.part_stride > 0, tmast = p.tmaps != nullptr;
+  const bool sx = sidx_on(c, chk, shard, tmast);
+  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk, eff_minblocks(c), full_row(c), sx, shard, tmast);
+  size_t smem = dyn_smem(c, sx);
   if (p.tmaps) smem = std::max(smem, (size_t)(kBlock / 32) * 8 * c->d * esize(c->odt));  // f4 staging (2 x 4 rows)
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
@@ -595,6 +612,12 @@ static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags,
   // (only without dynamic shared memory: a 0 % carve-out would cap residency at 1 CTA/SM)
   if (c->carveout >= 0 && smem == 0)
     CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, c->carveout));
+  // small rings (the SIDX id ring): the smallest carve-out that still fits the occupancy
+  // target (4 CTAs of smem + 1 KB driver reserve each), so the rest stays L1
+  if (c->carveout == 0 && smem > 0 && smem <= 8192) {
+    const int pct = (int)std::min<size_t>(100, (4 * (smem + 1024) * 100 + 233471) / 233472);
+    CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
+  }
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0) {
     CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem));
@@ -920,8 +943,9 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   i->epoch = c->epoch;
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0 && c->registered) {
-    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), c->sidx != 0);
-    const size_t smem = dyn_smem(c);
+    const bool sx = sidx_on(c, false, false, false);
+    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), sx);
+    const size_t smem = dyn_smem(c, sx);
     if (smem > 0) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem);
   }
@@ -951,6 +975,8 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
+  else if (!strcmp(key, "row_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "row_l2 not in [0, 5]"); c->row_l2 = (int)v; }
+  else if (!strcmp(key, "out_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "out_l2 not in [0, 5]"); c->out_l2 = (int)v; }
   else if (!strcmp(key, "tma_store")) c->tma_store = v ? 1 : 0;
   else if (!strcmp(key, "carveout")) {
     if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");

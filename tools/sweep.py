@@ -36,13 +36,14 @@ def main():
     tables, _ = SG.local_tables(w, 0, dev)
     layer = PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype)
     s = torch.cuda.Stream()
+    agg = {}
     for dist in a.dists.split(","):
         wd = synth.make_workload(a.config, G=1, dist=dist, **over)
         bs = [SG.rank_csr(wd, wd.batch_seed(i), 0, dev) for i in range(3)]
         nnz = np.mean([int(b[0][-1]) for b in bs])
         byt = nnz * (w.dim * w.elem_bytes() + 8) + w.T * w.B * (8 + w.dim * w.out_elem_bytes())
         for o in [o for _ in range(a.repeat) for o in a.opts]:
-            defaults = {"chunk_rows": 256, "minblocks": 0, "unroll": 0, "ctas_per_sm": 0, "stagger": 1, "sidx": 0, "carveout": 0, "fwd_interleave": 0, "tma_store": 0}
+            defaults = {"chunk_rows": 256, "minblocks": 0, "unroll": 0, "ctas_per_sm": 0, "stagger": 1, "sidx": 1, "carveout": 0, "fwd_interleave": 0, "tma_store": 0}
             kv = dict(defaults)
             for item in o.split(",") if o else []:
                 k, v = item.split("=")
@@ -69,10 +70,14 @@ def main():
                 clk = pw = None
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / a.steps
+            agg.setdefault((dist, o), []).append(ms)
             print(json.dumps({"config": a.config, "rows": int(w.rows[0]), "dist": dist, "opts": o, "ms": round(ms, 4),
                               "Msamples_s": round(w.B / ms / 1e3, 3), "GBs": round(byt / ms / 1e6, 1),
                               "sm_mhz": clk, "power_w": pw}), flush=True)
             assert layer.device_error() == 0
+    for (dist, o), v in agg.items():
+        print(json.dumps({"summary": True, "config": a.config, "dist": dist, "opts": o, "median_ms": round(float(np.median(v)), 4),
+                          "min_ms": round(min(v), 4), "n": len(v)}), flush=True)
     layer.close()
 
 
