@@ -123,6 +123,7 @@ struct emb_ctx {
   int bwd_interleave = 1;
   int fwd_interleave = 0;
   int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
+  int tail_div = 4;                // guided tail of the forward's chunk schedule
   int tma_store = 0;          // f4: stage pooled vectors, ship 4 per TMA scatter4
   void* d_tmaps = nullptr;    // f4: CUtensorMap [2 slots][kMaxG] of every rank's output slots
   float** d_dW = nullptr;
@@ -566,6 +567,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   p->stagger = c->stagger;
   p->interleave = c->fwd_interleave;
   p->row_l2 = c->row_l2;
+  p->tail_div = c->tail_div;
   p->out_l2 = c->out_l2;
   p->ctrl = c->ctrl;
   p->timeout_ns = c->timeout_ns;
@@ -975,6 +977,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
+  else if (!strcmp(key, "tail_div")) { if (v < 1 || v > 64) FAIL(c, EMB_ERR_ARG, "tail_div not in [1, 64]"); c->tail_div = (int)v; }
   else if (!strcmp(key, "row_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "row_l2 not in [0, 5]"); c->row_l2 = (int)v; }
   else if (!strcmp(key, "out_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "out_l2 not in [0, 5]"); c->out_l2 = (int)v; }
   else if (!strcmp(key, "tma_store")) c->tma_store = v ? 1 : 0;

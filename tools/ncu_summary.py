@@ -15,6 +15,9 @@ WANT = {
     "l1tex__t_sector_hit_rate.pct": "l1_hit_pct",
     "l1tex__throughput.avg.pct_of_peak_sustained_active": "l1_pct",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed": "sm_pct",
+    "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed": "l1_data_pipe_pct",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum": "l1_shared_wavefronts",
+    "smsp__issue_active.avg.pct_of_peak_sustained_active": "issue_pct",
     "sm__warps_active.avg.pct_of_peak_sustained_active": "occupancy_pct",
     "launch__registers_per_thread": "regs",
     "launch__grid_size": "grid",

@@ -28,6 +28,7 @@ def main():
     ap.add_argument("--opts", nargs="*", default=[""])
     ap.add_argument("--baseline", action="store_true")
     ap.add_argument("--repeat", type=int, default=1)
+    ap.add_argument("--gap", type=float, default=0.0, help="idle seconds before each measurement (clock recovery)")
     ap.add_argument("--rows", type=int, default=None, help="override rows per table (e.g. an L2-resident table)")
     a = ap.parse_args()
     dev = torch.device("cuda", 0)
@@ -43,7 +44,7 @@ def main():
         nnz = np.mean([int(b[0][-1]) for b in bs])
         byt = nnz * (w.dim * w.elem_bytes() + 8) + w.T * w.B * (8 + w.dim * w.out_elem_bytes())
         for o in [o for _ in range(a.repeat) for o in a.opts]:
-            defaults = {"chunk_rows": 256, "minblocks": 0, "unroll": 0, "ctas_per_sm": 0, "stagger": 1, "sidx": 1, "carveout": 0, "fwd_interleave": 0, "tma_store": 0}
+            defaults = {"chunk_rows": 256, "minblocks": 0, "unroll": 0, "ctas_per_sm": 0, "stagger": 1, "sidx": 1, "carveout": 0, "fwd_interleave": 0, "tma_store": 0, "tail_div": 4}
             kv = dict(defaults)
             for item in o.split(",") if o else []:
                 k, v = item.split("=")
@@ -55,6 +56,12 @@ def main():
             for i in range(5):
                 fn(i)
             torch.cuda.synchronize()
+            if a.gap > 0:
+                import time
+                time.sleep(a.gap)
+                for i in range(2):
+                    fn(i)
+                torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
             e0.record(s)
             for i in range(a.steps):
