@@ -29,6 +29,7 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402
 
+METRIC = "EMB fwd samples/sec at 1/2/4/8 B200 (max over ranks); % of HBM/NVLink roofline"   # BASELINE.json
 NVLINK_GBS = 770.0      # measured peer copy per direction (B200_PROFILING.md); nominal 900
 HBM_FALLBACK = 6650.0   # B200_PROFILING.md fallback if MEASURED_PEAKS.json is absent
 
@@ -251,7 +252,7 @@ def reference_arm(args):
         smp._pool.terminate()
     sec = float(np.mean(per_step))
     val = w.B / sec
-    line = {"impl": "reference", "metric": "EMB fwd samples/sec (max over ranks)", "value": val, "unit": "samples/s",
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "samples/s",
             "n_gpus": N, "steps": args.steps, "warmup": args.warmup, "ms_per_step": sec * 1e3,
             "higher_is_better": True, "scaling": "weak" if args.config.startswith("weak") else "strong",
             "vs_baseline": None, "dtype": "f32" if w.wdtype == "f32" else "bf16", "data": "synthetic",
@@ -562,7 +563,7 @@ def main():
     if N > 1:
         dist.barrier()
     if rank == 0:
-        line = {"metric": "EMB fwd samples/sec (max over ranks)", "value": value, "unit": "samples/s", "n_gpus": N,
+        line = {"metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                 "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None,
                 "dtype": "f32" if (w.wdtype == "f32") else "bf16", "data": "synthetic",
