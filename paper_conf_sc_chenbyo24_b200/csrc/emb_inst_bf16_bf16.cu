@@ -21,6 +21,8 @@ KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard, bool tmast
   }
   if (!full) return emb_fwd_kernel<VB, NV, WT, OT, 4, CHECK, 4, false>;  // rows narrower than a warp
   if constexpr (!CHECK && NV == 1) {
+    if (unroll == 3)  // experiment: 2 groups of 8 rows in flight per warp, 16 warps/SM (128 registers)
+      return sidx ? emb_fwd_kernel<VB, NV, WT, OT, 8, false, 2, true, true> : emb_fwd_kernel<VB, NV, WT, OT, 8, false, 2, true, false>;
     if (sidx && unroll == 4 && mb == 4) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, true>;
     if (sidx && unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, false, 6, true, true>;
   }

@@ -166,7 +166,7 @@ static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
   const int u = c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4);
   const int mb = c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1);
   return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
-         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && mb == 4) || u == 2);
+         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && mb == 4) || u == 2 || u == 3);
 }
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
 static size_t dyn_smem(const emb_ctx* c, bool sidx = false) {
@@ -966,8 +966,9 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "stagger")) c->stagger = v ? 1 : 0;
   else if (!strcmp(key, "timeout_ms")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "timeout_ms < 1"); c->timeout_ns = v * 1000000ll; }
   else if (!strcmp(key, "unroll")) {
-    if (v != 0 && v != 2 && v != 4 && v != 8 && v != 16 && v != -4 && v != -8 && v != -12 && v != -16)
-      FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline), 8, 16 (cp.async ring) or -4/-8/-12/-16 (ring v2)");
+    if (v != 0 && v != 2 && v != 3 && v != 4 && v != 8 && v != 16 && v != -4 && v != -8 && v != -12 && v != -16)
+      FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline), 3 (2 x 8 rows, 16 warps/SM), 8, 16 (cp.async ring) "
+                           "or -4/-8/-12/-16 (ring v2)");
     c->unroll = (int)v;
   }
   else if (!strcmp(key, "minblocks")) {
