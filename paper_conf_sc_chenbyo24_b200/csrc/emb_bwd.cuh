@@ -91,6 +91,8 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
   const bool active = lane < p.lanes;
   const int64_t rowbytes = (int64_t)p.d * 4;
   const int64_t B = p.B;
+  __shared__ __align__(16) uint32_t bwd_ring[kBlock / 32][128];     // per-warp id ring
+  const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(&bwd_ring[threadIdx.x >> 5][0]);
   // acquire every DP rank's dY of this epoch
   if (threadIdx.x == 0 && p.G > 1) wait_flags_geq(p.my_ready, p.G, p.rank, p.epoch, p.timeout_ns, &p.ctrl->err);
   __syncthreads();
@@ -123,24 +125,31 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
         while (b >= p.bstart[dst + 1]) ++dst;
         return p.gsrc[dst] + ((b - p.bstart[dst]) * p.T + tglob) * rowbytes + lane * VB;
       };
-      // Per bag: the bag's gradient vector (prefetched one bag ahead, with the bag's first
-      // 32 row ids) is added once per DISTINCT row of each 32-id slice, multiplied by the
+      // Per bag: the bag's gradient vector (prefetched one bag ahead) is added once per DISTINCT row of each 32-id slice, multiplied by the
       // row's multiplicity (match.any): zipf-hot rows repeat inside a bag, and fewer
       // atomics on the same L2 address is what bounds this kernel.
       auto bag_start = [&](int bag) -> int64_t { return __shfl_sync(kFull, o_l, bag); };
-      auto load_ids = [&](int64_t from, int64_t to) -> uint32_t {
-        return (from + lane < to) ? (uint32_t)ld_stream_i64(p.indices + from + lane) : (0x80000000u | lane);
+      // The chunk's row ids stream through a per-warp shared-memory ring of 4 batches of 32
+      // (cp.async of each int64 id's low word, up to 3 batches ahead of the slice being
+      // scattered), so no slice waits on an id load from DRAM.
+      const int64_t pos0 = bag_start(0);
+      const int32_t nrel = (int32_t)(bag_start(nb) - pos0);
+      const int64_t* ip = p.indices + pos0;
+      const int32_t nbatch = (nrel + 31) >> 5;
+      int32_t fetched = 0;
+      auto fetch = [&]() {
+        const int32_t at = fetched * 32 + lane;
+        if (at < nrel)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(ring_s + (uint32_t)(((fetched & 3) * 32 + lane) * 4)),
+                       "l"(ip + at) : "memory");
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        ++fetched;
       };
       uint32_t gn[NV][W];
-      uint32_t xn = 0;
-      {
-        const int64_t s0 = bag_start(0), e0 = bag_start(1);
-        xn = load_ids(s0, e0);
-        if (active) {
-          const char* a = gaddr(0);
+      if (active && nb > 0) {
+        const char* a = gaddr(0);
 #pragma unroll
-          for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
-        }
+        for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
       }
       for (int bag = 0; bag < nb; ++bag) {
         uint32_t g[NV][W];
@@ -148,19 +157,26 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
         for (int v = 0; v < NV; ++v)
 #pragma unroll
           for (int i = 0; i < W; ++i) g[v][i] = gn[v][i];
-        uint32_t x = xn;
         const int64_t s0 = bag_start(bag), e0 = bag_start(bag + 1);
-        if (bag + 1 < nb) {                               // next bag: gradient + first ids in flight
-          const int64_t s1 = e0, e1 = bag_start(bag + 2 > 31 ? 31 : bag + 2);
-          xn = load_ids(s1, bag + 1 < nb ? e1 : s1);
-          if (active) {
-            const char* a = gaddr(bag + 1);
+        if (bag + 1 < nb && active) {                     // next bag's gradient in flight
+          const char* a = gaddr(bag + 1);
 #pragma unroll
-            for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
-          }
+          for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, gn[v]);
         }
         for (int64_t c0 = s0; c0 < e0; c0 += 32) {
-          if (c0 != s0) x = load_ids(c0, e0);
+          const int32_t r0 = (int32_t)(c0 - pos0);
+          const int32_t lo = r0 >> 5, hi = min((r0 + 31) >> 5, nbatch - 1);
+          while (fetched < nbatch && fetched <= lo + 3) fetch();
+          switch (min(fetched - 1 - hi, 3)) {             // batches lo..hi landed
+            case 0: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
+            case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+            case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+            default: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+          }
+          __syncwarp();
+          uint32_t x = 0x80000000u | lane;
+          if (c0 + lane < e0)
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(ring_s + (uint32_t)(((r0 + lane) & 127) * 4)) : "memory");
           const unsigned same = __match_any_sync(kFull, x);
           const bool lead = (x & 0x80000000u) == 0 && (__ffs(same) - 1) == lane;
           unsigned leaders = __ballot_sync(kFull, lead);
@@ -183,6 +199,8 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
           }
         }
       }
+      asm volatile("cp.async.wait_group 0;" ::: "memory");   // no copy outlives the chunk
+      __syncwarp();
     }
   }
   // completion: every CTA's reads of peer slots are done before the last CTA tells the
