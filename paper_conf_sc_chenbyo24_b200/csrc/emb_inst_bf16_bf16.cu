@@ -70,4 +70,6 @@ KernelFn pick_tile_bf16_bf16(int vb, int nv, int unroll, bool check, int mb, boo
     default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
   }
 }
+// dual-stream kernel for 256-B rows (two half-warp bag streams per warp)
+KernelFn pick_ds_bf16_bf16(int mb) { return mb == 3 ? emb_fwd_ds_kernel<__nv_bfloat16, __nv_bfloat16, 3> : emb_fwd_ds_kernel<__nv_bfloat16, __nv_bfloat16, 4>; }
 }  // namespace emb

@@ -70,4 +70,6 @@ KernelFn pick_tile_f32_f32(int vb, int nv, int unroll, bool check, int mb, bool 
     default: return pick_c<16, 1, WT, OT>(unroll, check, mb, full, sidx, shard, tmast);
   }
 }
+// dual-stream kernel for 256-B rows (two half-warp bag streams per warp)
+KernelFn pick_ds_f32_f32(int mb) { return mb == 3 ? emb_fwd_ds_kernel<float, float, 3> : emb_fwd_ds_kernel<float, float, 4>; }
 }  // namespace emb

@@ -95,7 +95,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 1, carveout = 0;  // 0: auto per tile
+  int chunk_rows = 256, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 1, carveout = 0, ds = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -167,6 +167,16 @@ static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
   const int mb = c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1);
   return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
          (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && mb == 4) || u == 2 || u == 3);
+}
+// dual-stream kernel (emb_fwd_ds_kernel): 256-B rows, default options, no bounds check,
+// no row shards, direct stores
+static bool ds_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
+  return c->ds != 0 && c->unroll == 0 && c->minblocks == 0 && !check && !shard && !tmast &&
+         (int64_t)c->d * (int64_t)esize(c->wdt) == 256;
+}
+static KernelFn pick_ds(emb_dtype_t w, emb_dtype_t o, int mb) {
+  if (w == EMB_F32) return o == EMB_F32 ? pick_ds_f32_f32(mb) : pick_ds_f32_bf16(mb);
+  return o == EMB_F32 ? pick_ds_bf16_f32(mb) : pick_ds_bf16_bf16(mb);
 }
 // shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
 static size_t dyn_smem(const emb_ctx* c, bool sidx = false) {
@@ -463,6 +473,7 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
       cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
                                             full, false, false));
     }
+    if (c->d * (int64_t)esize(c->wdt) == 256) cudaFuncGetAttributes(&a, pick_ds(c->wdt, c->odt, c->ds));
     cudaFuncGetAttributes(&a, emb_wait_kernel);
     cudaFuncGetAttributes(&a, emb_unpack_kernel);
     cudaFuncGetAttributes(&a, emb_unpack8_kernel);
@@ -605,8 +616,10 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
   const bool chk = (flags & EMB_FWD_CHECK_BOUNDS) != 0, shard = p.part_stride > 0, tmast = p.tmaps != nullptr;
   const bool sx = sidx_on(c, chk, shard, tmast);
-  KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk, eff_minblocks(c), full_row(c), sx, shard, tmast);
-  size_t smem = dyn_smem(c, sx);
+  const bool ds = ds_on(c, chk, shard, tmast);
+  KernelFn k = ds ? pick_ds(c->wdt, c->odt, c->ds)
+                  : pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk, eff_minblocks(c), full_row(c), sx, shard, tmast);
+  size_t smem = ds ? (size_t)(kBlock / 32) * 1024 : dyn_smem(c, sx);   // ds: two 512-B id rings per warp
   if (p.tmaps) smem = std::max(smem, (size_t)(kBlock / 32) * 8 * c->d * esize(c->odt));  // f4 staging (2 x 4 rows)
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
@@ -946,8 +959,10 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0 && c->registered) {
     const bool sx = sidx_on(c, false, false, false);
-    KernelFn k = pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), sx);
-    const size_t smem = dyn_smem(c, sx);
+    const bool ds = ds_on(c, false, false, false);
+    KernelFn k = ds ? pick_ds(c->wdt, c->odt, c->ds)
+                    : pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), sx);
+    const size_t smem = ds ? (size_t)(kBlock / 32) * 1024 : dyn_smem(c, sx);
     if (smem > 0) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem);
   }
@@ -976,6 +991,10 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->minblocks = (int)v;
   }
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
+  else if (!strcmp(key, "ds")) {
+    if (v != 0 && v != 1 && v != 3 && v != 4) FAIL(c, EMB_ERR_ARG, "ds must be 0 (off, default), 1 or 4 (4 CTAs/SM), 3 (3 CTAs/SM)");
+    c->ds = (int)v;
+  }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "tail_div")) { if (v < 1 || v > 64) FAIL(c, EMB_ERR_ARG, "tail_div not in [1, 64]"); c->tail_div = (int)v; }

@@ -336,7 +336,8 @@ VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),
 @pytest.mark.parametrize("opts", [{"unroll": 2}, {"unroll": 4}, {"unroll": 8}, {"unroll": 16},
                                   {"unroll": 4, "minblocks": 1}, {"unroll": 4, "minblocks": 6},
                                   {"chunk_rows": 1}, {"chunk_rows": 100000}, {"stagger": 0}, {"sidx": 0},
-                                  {"sidx": 0, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}, {"sidx": 0, "chunk_rows": 7}, {"fwd_interleave": 1},
+                                  {"sidx": 0, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}, {"sidx": 0, "chunk_rows": 7},
+                                  {"ds": 1}, {"ds": 3}, {"ds": 1, "chunk_rows": 3}, {"ds": 1, "tail_div": 1}, {"fwd_interleave": 1},
                                   {"tma_store": 1}, {"tma_store": 1, "chunk_rows": 3}, {"unroll": -8}, {"unroll": -16},
                                   {"unroll": -12, "chunk_rows": 5}])
 @pytest.mark.parametrize("case", range(len(VARIANT_CASES)))
