@@ -568,6 +568,10 @@ def main():
                 "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None,
                 "dtype": "f32" if (w.wdtype == "f32") else "bf16", "data": "synthetic",
                 "config": config_desc(w, N), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "pooled_vectors_per_s": w.B * w.T / (ms * 1e-3),
+                "scaling_note": "table-wise model parallelism: each GPU adds its tables AND (weak) its 16,384 samples, so "
+                                "every GPU pools its tables for the whole global batch; ideal samples/s is flat in N, "
+                                "pooled_vectors_per_s (samples x tables) is the quantity that ideally grows with N",
                 "gpu_launches": args.steps, "clocks": clk.summary(), **extra}
         print(json.dumps(line), flush=True)
     if N > 1:
