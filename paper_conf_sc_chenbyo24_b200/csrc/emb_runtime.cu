@@ -166,7 +166,7 @@ static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
   const int u = c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4);
   const int mb = c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1);
   return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
-         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && mb == 4) || u == 2 || u == 3);
+         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && (mb == 4 || mb == 5)) || u == 2 || u == 3);
 }
 // dual-stream kernel (emb_fwd_ds_kernel): 256-B rows, default options, no bounds check,
 // no row shards, direct stores
@@ -630,7 +630,8 @@ static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags,
   // small rings (the SIDX id ring): the smallest carve-out that still fits the occupancy
   // target (4 CTAs of smem + 1 KB driver reserve each), so the rest stays L1
   if (c->carveout == 0 && smem > 0 && smem <= 8192) {
-    const int pct = (int)std::min<size_t>(100, (4 * (smem + 1024) * 100 + 233471) / 233472);
+    const size_t want = (size_t)std::max(4, eff_minblocks(c));   // occupancy target (CTAs/SM)
+    const int pct = (int)std::min<size_t>(100, (want * (smem + 1024) * 100 + 233471) / 233472);
     CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
   }
   int per_sm = c->ctas_per_sm;
@@ -987,7 +988,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->unroll = (int)v;
   }
   else if (!strcmp(key, "minblocks")) {
-    if (v != 0 && v != 1 && v != 4 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4 or 6");
+    if (v != 0 && v != 1 && v != 4 && v != 5 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4, 5 or 6");
     c->minblocks = (int)v;
   }
   else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
