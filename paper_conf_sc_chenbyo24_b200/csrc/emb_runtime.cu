@@ -183,7 +183,7 @@ static size_t dyn_smem(const emb_ctx* c, bool sidx = false) {
   if (eff_unroll(c) < 0 && c->nv == 1 && full_row(c) && !c->has_shard)  // ring v2: R rows of 512 B per warp
     return (size_t)(kBlock / 32) * (size_t)(-eff_unroll(c) == 4 ? 8 : -eff_unroll(c)) * 32 * c->vb;
   if (eff_unroll(c) >= 8 && c->nv == 1) return (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb;
-  if (sidx) return (size_t)(kBlock / 32) * 512;   // id ring: 4 x 32 x 4 B per warp
+  if (sidx) return (size_t)(kBlock / 32) * EMB_SIDX_RING * 128;   // id ring: EMB_SIDX_RING x 32 x 4 B per warp
   return 0;
 }
 
