@@ -117,6 +117,7 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
       const int64_t o_l = (lane <= nb) ? ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane) : 0;
       const TableDesc* tdp = p.tables + t_l;
       const int64_t tglob = __ldg(&tdp->tglob);
+      const bool pack = __ldg(reinterpret_cast<const long long*>(&tdp->rows)) < (1ll << 26);
       char* dwl = reinterpret_cast<char*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t_l))) + lane * VB;
 
       auto gaddr = [&](int bag) -> const char* {        // dY[b][tglob] on the DP rank owning b
@@ -180,12 +181,16 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
           const unsigned same = __match_any_sync(kFull, x);
           const bool lead = (x & 0x80000000u) == 0 && (__ffs(same) - 1) == lane;
           unsigned leaders = __ballot_sync(kFull, lead);
+          // row id and multiplicity travel in one word (ids < 2^26): one SHFL per distinct
+          // row instead of two -- the leader loop is bound by the MIO pipe
+          const uint32_t xm = pack ? (x | ((uint32_t)__popc(same) << 26)) : x;
           const float mult = (float)__popc(same);
           while (leaders) {
             const int l = __ffs(leaders) - 1;
             leaders &= leaders - 1;
-            const uint32_t xl = __shfl_sync(kFull, x, l);
-            const float m = __shfl_sync(kFull, mult, l);
+            const uint32_t v = __shfl_sync(kFull, xm, l);
+            const uint32_t xl = pack ? (v & 0x03ffffffu) : v;
+            const float m = pack ? (float)(v >> 26) : __shfl_sync(kFull, mult, l);
             if (active) {
               char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
 #pragma unroll
