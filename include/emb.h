@@ -196,7 +196,12 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * warp in shared memory and shipped 4 at a time to 4 arbitrary output rows with one TMA
  * scatter4; needs full-warp rows with one vector per lane and d <= 256),
  * "enable_backward" (f2: 1 before emb_register_tables adds two fp32 grad slots
- * [B_r][T][d] to the symmetric buffer for emb_backward),
+ * [B_r][T][d] to the symmetric buffer for emb_backward), f2 backward tunables:
+ * "bwd_interleave" (1 = chunks interleaved across tables, default; 0 = table-major),
+ * "bwd_group" (tables interleaved at a time, default 4; 0 = all local tables),
+ * "bwd_v2" (1 = distinct rows of a slice scattered from a compacted shared-memory list,
+ * default), "bwd_cache" (per-warp shared-memory dW row cache slots: 0, 8, 16 (default)
+ * or 32; needs bwd_v2 and one vector per lane), "bwd_chunk_rows" (0 = chunk_rows),
  * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
  * of that many records and makes every warp append {globaltimer ns, bytes stored to
  * peers << 32 | bytes stored locally} after each claimed chunk; 0 disables).
@@ -214,7 +219,8 @@ emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
  *   emb_backward(ctx, offsets, indices, dW, flags, stream) -> one fused kernel acquires
  *       every peer's "ready" flag and, per local bag, loads the
  *       bag's gradient vector from the DP rank's slot (one-sided NVLink load) and
- *       atomically adds it (red.add.f32, FTZ per the hardware atomic) into the rows of
+ *       atomically adds it (red.add.f32, FTZ per the hardware atomic; a warp may first
+ *       sum a hot row's contributions of one chunk in shared memory) into the rows of
  *       dW[t_l] (caller-owned device fp32 [M_t][d], NOT zeroed by the library; 16-byte
  *       aligned) for every index of the bag.  Same CSR as emb_forward.  Accumulation
  *       order is unspecified (atomics): results match the oracle within the fp32

@@ -35,7 +35,7 @@ struct BwdParams {
   Ctrl* ctrl;                  // uses bwork / bdone
   int64_t timeout_ns;
   int32_t T, T_r, d, G, rank, lanes, chunk_rows;
-  int32_t interleave;          // 1: chunk c -> table c mod T_r (spreads same-row atomics over time)
+  int32_t interleave;          // table group size g: chunks interleaved over g tables at a time (1 = table-major)
   uint32_t epoch;
 };
 
@@ -84,14 +84,35 @@ __device__ __forceinline__ bool wait_flags_geq(const uint32_t* flags, int G, int
 }
 
 // VB bytes per lane vector, NV vectors per lane (row = 32*VB*NV bytes when all lanes active)
-template <int VB, int NV>
+// V2: each slice's distinct rows are compacted into a per-warp shared-memory list (row id
+// and multiplicity in one word) and scattered from it with broadcast LDS.128 reads, 8
+// REDs per iteration -- no SHFL / find-first-set chain per distinct row
+//
+// HC > 0 (needs V2): each warp privatizes up to HC dW rows of its current chunk in shared
+// memory (direct-mapped by a multiplicative hash of the row id, first come first served,
+// a row whose slot is taken goes straight to L2).  A zipf-hot row then costs one RED per
+// chunk (the flush at the chunk's end) instead of one per bag slice: same-address
+// atomics on the hottest rows are what serialize in the L2.
+template <int VB, int NV, bool V2 = false, int HC = 0>
 __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__ BwdParams p) {
+  static_assert(HC == 0 || (V2 && HC <= 32 && (HC & (HC - 1)) == 0), "cache: V2, power of two <= 32 slots");
   constexpr int W = VB / 4;
   const int lane = threadIdx.x & 31;
   const bool active = lane < p.lanes;
   const int64_t rowbytes = (int64_t)p.d * 4;
   const int64_t B = p.B;
   __shared__ __align__(16) uint32_t bwd_ring[kBlock / 32][128];     // per-warp id ring
+  __shared__ __align__(16) uint32_t bwd_list[V2 ? kBlock / 32 : 1][V2 ? 80 : 4];  // V2: compacted (id|mult) + mult
+  const uint32_t list_s = (uint32_t)__cvta_generic_to_shared(&bwd_list[V2 ? (threadIdx.x >> 5) : 0][0]);
+  // HC: per-warp row cache [HC][32*VB*NV bytes] + tags [HC] in dynamic shared memory
+  constexpr uint32_t kRowB = 32u * VB * NV;
+  constexpr uint32_t kEmpty = 0xffffffffu;
+  constexpr int kLogHC = HC >= 32 ? 5 : HC >= 16 ? 4 : HC >= 8 ? 3 : HC >= 4 ? 2 : HC >= 2 ? 1 : 0;
+  extern __shared__ __align__(16) unsigned char bwd_dyn[];
+  const uint32_t cache_s = HC ? (uint32_t)__cvta_generic_to_shared(bwd_dyn) + (threadIdx.x >> 5) * (HC * (kRowB + 4u)) : 0u;
+  const uint32_t tag_s = cache_s + HC * kRowB;
+  if (HC > 0 && lane < HC) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * lane), "r"(kEmpty) : "memory");
+  __syncwarp();
   const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(&bwd_ring[threadIdx.x >> 5][0]);
   // acquire every DP rank's dY of this epoch
   if (threadIdx.x == 0 && p.G > 1) wait_flags_geq(p.my_ready, p.G, p.rank, p.epoch, p.timeout_ns, &p.ctrl->err);
@@ -111,8 +132,22 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
       if ((int64_t)c >= nchunks) break;
       // interleave tables (chunk c -> table c mod T_r): a zipf-hot dW row then receives its
       // atomics spread over the whole kernel instead of from every warp at once
-      const int t_l = p.interleave ? (int)(c % p.T_r) : (int)(c / cpt);
-      const int64_t b0 = (p.interleave ? (int64_t)(c / p.T_r) : (int64_t)c % cpt) * cb;
+      // (in groups of g tables: the touched dW rows of g tables stay live in L2 at once)
+      const int g = p.interleave, nfull = p.T_r / g;
+      const int64_t nfc = (int64_t)nfull * g * cpt;       // chunks of the full groups
+      int t_l;
+      int64_t bi;
+      if ((int64_t)c < nfc) {
+        const int64_t r = (int64_t)c % ((int64_t)g * cpt);
+        t_l = (int)((int64_t)c / ((int64_t)g * cpt)) * g + (int)(r % g);
+        bi = r / g;
+      } else {                                            // the last, smaller group
+        const int rem = p.T_r - nfull * g;
+        const int64_t r = (int64_t)c - nfc;
+        t_l = nfull * g + (int)(r % rem);
+        bi = r / rem;
+      }
+      const int64_t b0 = bi * cb;
       const int nb = (int)min((int64_t)cb, B - b0);
       const int64_t o_l = (lane <= nb) ? ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane) : 0;
       const TableDesc* tdp = p.tables + t_l;
@@ -184,6 +219,77 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
           // row id and multiplicity travel in one word (ids < 2^26): one SHFL per distinct
           // row instead of two -- the leader loop is bound by the MIO pipe
           const uint32_t xm = pack ? (x | ((uint32_t)__popc(same) << 26)) : x;
+          if constexpr (V2) {
+            const int n = __popc(leaders);
+            if (lead) {
+              const uint32_t at = list_s + 4u * (uint32_t)__popc(leaders & ((1u << lane) - 1u));
+              asm volatile("st.shared.u32 [%0], %1;" ::"r"(at), "r"(xm) : "memory");
+              if (!pack) asm volatile("st.shared.u32 [%0], %1;" ::"r"(at + 160u), "r"((uint32_t)__popc(same)) : "memory");
+            }
+            __syncwarp();
+            for (int k = 0; k < n; k += 8) {
+              uint32_t wv[8], mv[8];
+              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
+                           : "r"(list_s + 4u * k) : "memory");
+              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[4]), "=r"(wv[5]), "=r"(wv[6]), "=r"(wv[7])
+                           : "r"(list_s + 4u * k + 16u) : "memory");
+              if (!pack) {
+                asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[0]), "=r"(mv[1]), "=r"(mv[2]), "=r"(mv[3])
+                             : "r"(list_s + 4u * k + 160u) : "memory");
+                asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[4]), "=r"(mv[5]), "=r"(mv[6]), "=r"(mv[7])
+                             : "r"(list_s + 4u * k + 176u) : "memory");
+              }
+#pragma unroll
+              for (int u = 0; u < 8; ++u) {
+                if constexpr (HC > 0) {
+                  if (k + u < n) {
+                    const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
+                    const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
+                    const uint32_t h = HC == 1 ? 0u : (xl * 2654435761u) >> (32 - kLogHC);
+                    uint32_t tg;
+                    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * h) : "memory");
+                    const bool hit = tg == xl, claim = tg == kEmpty;
+                    if (claim) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * h), "r"(xl) : "memory");
+                    if (active) {
+#pragma unroll
+                      for (int v = 0; v < NV; ++v) {
+                        uint32_t gm[W];
+#pragma unroll
+                        for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
+                        const uint32_t sa = cache_s + h * kRowB + (uint32_t)(v * 32 + lane) * VB;
+                        if (hit) {                            // this lane's columns only: no atomics
+                          uint32_t cv[W];
+                          lds_bytes<VB>(sa, cv);
+#pragma unroll
+                          for (int i = 0; i < W; ++i) cv[i] = __float_as_uint(__uint_as_float(cv[i]) + __uint_as_float(gm[i]));
+                          sts_bytes<VB>(sa, cv);
+                        } else if (claim) {
+                          sts_bytes<VB>(sa, gm);
+                        } else {
+                          red_add_vec<VB>(reinterpret_cast<float*>(dwl + (uint64_t)xl * (uint64_t)rowbytes + v * 32 * VB), gm);
+                        }
+                      }
+                    }
+                  }
+                  continue;
+                }
+                if (k + u < n && active) {
+                  const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
+                  const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
+                  char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
+#pragma unroll
+                  for (int v = 0; v < NV; ++v) {
+                    uint32_t gm[W];
+#pragma unroll
+                    for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
+                    red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), gm);
+                  }
+                }
+              }
+            }
+            __syncwarp();                                 // the list is rewritten by the next slice
+            continue;
+          }
           const float mult = (float)__popc(same);
           while (leaders) {
             const int l = __ffs(leaders) - 1;
@@ -206,6 +312,26 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
       }
       asm volatile("cp.async.wait_group 0;" ::: "memory");   // no copy outlives the chunk
       __syncwarp();
+      if constexpr (HC > 0) {                             // flush the chunk's cached rows
+        uint32_t tg = kEmpty;
+        if (lane < HC) asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * lane) : "memory");
+        unsigned occ = __ballot_sync(kFull, tg != kEmpty);
+        while (occ) {
+          const int l = __ffs(occ) - 1;
+          occ &= occ - 1;
+          const uint32_t xl = __shfl_sync(kFull, tg, l);
+          if (active) {
+#pragma unroll
+            for (int v = 0; v < NV; ++v) {
+              uint32_t cv[W];
+              lds_bytes<VB>(cache_s + (uint32_t)l * kRowB + (uint32_t)(v * 32 + lane) * VB, cv);
+              red_add_vec<VB>(reinterpret_cast<float*>(dwl + (uint64_t)xl * (uint64_t)rowbytes + v * 32 * VB), cv);
+            }
+          }
+        }
+        if (lane < HC) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * lane), "r"(kEmpty) : "memory");
+        __syncwarp();
+      }
     }
   }
   // completion: every CTA's reads of peer slots are done before the last CTA tells the

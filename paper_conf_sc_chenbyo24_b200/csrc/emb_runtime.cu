@@ -121,6 +121,10 @@ struct emb_ctx {
   uint64_t bepoch = 0;
   bool bwd_ready_pending = false;
   int bwd_interleave = 1;
+  int bwd_v2 = 1;                  // backward slice scatter from a compacted smem list
+  int bwd_cache = 16;              // per-warp dW row cache slots (0 off; 8 / 16 / 32; needs bwd_v2)
+  int bwd_chunk_rows = 0;          // backward chunk target rows (0: chunk_rows)
+  int bwd_group = 4;               // tables interleaved at a time in the backward (0: all T_r)
   int fwd_interleave = 0;
   int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
   int tail_div = 4;                // guided tail of the forward's chunk schedule
@@ -485,6 +489,16 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2, true>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4, true>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 8>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 16>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 32>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 8>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 16>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 32>);
     cudaGetLastError();
   }
   return EMB_OK;
@@ -805,8 +819,10 @@ static void fill_bwd_params(emb_ctx_t* c, BwdParams* p) {
   p->G = c->G;
   p->rank = c->rank;
   p->lanes = c->blanes;
-  p->chunk_rows = c->chunk_rows;
-  p->interleave = c->bwd_interleave;
+  p->chunk_rows = c->bwd_chunk_rows > 0 ? c->bwd_chunk_rows : c->chunk_rows;
+  // chunk order: table groups of `bwd_group` tables, chunks interleaved inside a group
+  // (1 = table-major, T_r = every table interleaved)
+  p->interleave = c->bwd_interleave ? ((c->bwd_group > 0 && c->bwd_group < c->T_r) ? c->bwd_group : std::max(c->T_r, 1)) : 1;
   p->epoch = (uint32_t)c->bepoch;
 }
 
@@ -867,13 +883,27 @@ emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* i
   p.offsets = offsets;
   p.indices = indices;
   void (*k)(BwdParams) = nullptr;
-  if (c->bvb == 8) k = emb_bwd_kernel<8, 1>;
+  size_t smem = 0;
+  const bool cache_ok = c->bnv == 1;                  // cache variants: 256-B and 512-B rows
+  if (c->bwd_v2 && c->bwd_cache && cache_ok) {
+    const bool w16 = c->bvb == 16;
+    if (c->bwd_cache == 8) k = w16 ? emb_bwd_kernel<16, 1, true, 8> : emb_bwd_kernel<8, 1, true, 8>;
+    else if (c->bwd_cache == 16) k = w16 ? emb_bwd_kernel<16, 1, true, 16> : emb_bwd_kernel<8, 1, true, 16>;
+    else k = w16 ? emb_bwd_kernel<16, 1, true, 32> : emb_bwd_kernel<8, 1, true, 32>;
+    smem = (size_t)(kBlock / 32) * c->bwd_cache * (32 * c->bvb + 4);
+    CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  } else if (c->bwd_v2) {
+    if (c->bvb == 8) k = emb_bwd_kernel<8, 1, true>;
+    else if (c->bnv == 2) k = emb_bwd_kernel<16, 2, true>;
+    else if (c->bnv == 4) k = emb_bwd_kernel<16, 4, true>;
+    else k = emb_bwd_kernel<16, 1, true>;
+  } else if (c->bvb == 8) k = emb_bwd_kernel<8, 1>;
   else if (c->bnv == 2) k = emb_bwd_kernel<16, 2>;
   else if (c->bnv == 4) k = emb_bwd_kernel<16, 4>;
   else k = emb_bwd_kernel<16, 1>;
   int per_sm = 0;
-  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, 0));
-  k<<<c->num_sms * std::max(per_sm, 1), kBlock, 0, s>>>(p);
+  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem));
+  k<<<c->num_sms * std::max(per_sm, 1), kBlock, smem, s>>>(p);
   CK(c, cudaGetLastError());
   return EMB_OK;
 }
@@ -997,6 +1027,13 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->ds = (int)v;
   }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
+  else if (!strcmp(key, "bwd_v2")) c->bwd_v2 = v ? 1 : 0;
+  else if (!strcmp(key, "bwd_cache")) {
+    if (v != 0 && v != 8 && v != 16 && v != 32) FAIL(c, EMB_ERR_ARG, "bwd_cache must be 0, 8, 16 or 32");
+    c->bwd_cache = (int)v;
+  }
+  else if (!strcmp(key, "bwd_chunk_rows")) { if (v < 0 || v > 65536) FAIL(c, EMB_ERR_ARG, "bwd_chunk_rows not in [0, 65536]"); c->bwd_chunk_rows = (int)v; }
+  else if (!strcmp(key, "bwd_group")) { if (v < 0 || v > 4096) FAIL(c, EMB_ERR_ARG, "bwd_group not in [0, 4096]"); c->bwd_group = (int)v; }
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "tail_div")) { if (v < 1 || v > 64) FAIL(c, EMB_ERR_ARG, "tail_div not in [1, 64]"); c->tail_div = (int)v; }
   else if (!strcmp(key, "row_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "row_l2 not in [0, 5]"); c->row_l2 = (int)v; }

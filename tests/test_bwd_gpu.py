@@ -14,6 +14,7 @@ import emb_test_helpers as H
 import synth
 from oracle import emb_oracle as O
 from paper_conf_sc_chenbyo24_b200.comm import LocalGroup, run_ranks
+from paper_conf_sc_chenbyo24_b200 import emb as E
 from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
 
 DEV = torch.device("cuda", 0)
@@ -27,7 +28,7 @@ def _dY(w, seed, integer):
     return [rng.standard_normal((counts[r], w.T, w.dim)).astype(np.float32) for r in range(w.G)]
 
 
-def _run_bwd(w, dY, seed, epochs=1, flags=0):
+def _run_bwd(w, dY, seed, epochs=1, flags=0, opts=None):
     tabs = H.np_tables(w)
     offs, idxs = H.np_csrs(w, seed)
     tdev = [[torch.from_numpy(tabs[int(w.phys[t])]).to(DEV) for t in w.local_tables(r)] for r in range(w.G)]
@@ -38,6 +39,9 @@ def _run_bwd(w, dY, seed, epochs=1, flags=0):
         layers = run_ranks(w.G, lambda r: PgasEmbedding(r, w.G, 0, w.rows, w.owner, w.dim, tdev[r], w.B,
                                                         allgather=grp.allgather_for(r), backward=True))
     try:
+        for k, v in (opts or {}).items():
+            for L in layers:
+                E.emb_set_option(L.ctx, k, v)
         dW = [[torch.zeros((int(w.rows[t]), w.dim), device=DEV) for t in w.local_tables(r)] for r in range(w.G)]
         streams = [torch.cuda.Stream() for _ in range(w.G)]
         ins = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(w.G)]
@@ -97,3 +101,38 @@ def test_bwd_placement_invariance():
     for d in outs[1:]:
         for t in d:
             assert np.array_equal(d[t], outs[0][t])
+
+
+@pytest.mark.parametrize("opts", [{"bwd_interleave": 0}, {"bwd_group": 2}, {"bwd_group": 3}, {"bwd_group": 4},
+                                  {"bwd_group": 7}, {"bwd_group": 1}, {"bwd_v2": 1}, {"bwd_v2": 1, "bwd_group": 3},
+                                  {"bwd_v2": 1, "bwd_interleave": 0}, {"bwd_v2": 1, "bwd_cache": 8},
+                                  {"bwd_v2": 1, "bwd_cache": 16, "bwd_chunk_rows": 1024},
+                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}])
+def test_bwd_chunk_orders_integer_exact(opts):
+    """every chunk order (table-major, groups of g tables incl. a ragged last group, all
+    tables interleaved) visits every bag exactly once: exact on integer gradients"""
+    w = synth.make_workload("tiny", G=2, pmin=0, pmax=40, B=97, T=7, dim=64, rows=300, dist="zipf")
+    dY = _dY(w, 5, integer=True)
+    got, offs, idxs = _run_bwd(w, dY, 14, opts=opts)
+    ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    for t in range(w.T):
+        assert np.array_equal(got[t].astype(np.float64), ref[t]), t
+
+
+@pytest.mark.parametrize("dim,cache", [(16, 8), (64, 16), (128, 32), (256, 8)])
+def test_bwd_row_cache_exact_and_float_bound(dim, cache):
+    """f2 per-warp dW row cache (bwd_cache): integer gradients exact, float gradients within
+    the order-independent summation bound (cached rows are summed in shared memory first)"""
+    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512}
+    w = synth.make_workload("tiny", G=2, pmin=0, pmax=60, B=150, T=3, dim=dim, rows=200, dist="zipf")
+    got, offs, idxs = _run_bwd(w, _dY(w, 21, integer=True), 22, opts=opts)
+    ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, _dY(w, 21, integer=True), w.B, w.G)
+    for t in range(w.T):
+        assert np.array_equal(got[t].astype(np.float64), ref[t]), t
+    dY = _dY(w, 23, integer=False)
+    got, offs, idxs = _run_bwd(w, dY, 24, epochs=2, opts=opts)
+    ref, S, cnt = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    for t in range(w.T):
+        n = 2 * cnt[t][:, None]
+        err = np.abs(got[t].astype(np.float64) - 2 * ref[t])
+        assert np.all(err <= n * 2.0 ** -24 * 2 * S[t] + 1e-30), t
