@@ -67,6 +67,7 @@ typedef enum { EMB_F32 = 0, EMB_BF16 = 1 } emb_dtype_t;
 /* sticky device error word bits (emb_query_device_error) */
 #define EMB_DEVERR_TIMEOUT 0x1u
 #define EMB_DEVERR_BOUNDS 0x2u
+#define EMB_DEVERR_CAPACITY 0x4u /* emb_backward (bwd_algo 1): more lookups than the entry workspace; step skipped */
 
 /* All-gather over the caller's process group.  send: `bytes` bytes of this rank;
  * recv: world_size*bytes, rank order.  Return 0 on success.  Called only from
@@ -202,6 +203,11 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * "bwd_v2" (1 = distinct rows of a slice scattered from a compacted shared-memory list,
  * default), "bwd_cache" (per-warp shared-memory dW row cache slots: 0, 8, 16 (default)
  * or 32; needs bwd_v2 and one vector per lane), "bwd_chunk_rows" (0 = chunk_rows),
+ * "bwd_algo" (0 = atomic scatter per bag slice; 1 = counting sort of the lookups by dW
+ * row + segmented gather-sum, one red.add per run of equal rows: library-owned workspace
+ * of 4 B per local row + 8 B per lookup, sized on the first call from the CSR (one host
+ * sync) or preset by "bwd_max_nnz"; a later CSR with more lookups sets
+ * EMB_DEVERR_CAPACITY and skips the step),
  * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
  * of that many records and makes every warp append {globaltimer ns, bytes stored to
  * peers << 32 | bytes stored locally} after each claimed chunk; 0 disables).

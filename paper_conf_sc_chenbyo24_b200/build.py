@@ -22,7 +22,7 @@ CSRC = os.path.join(PKG, "csrc")
 LIBS = {
     "emb": dict(srcs=[os.path.join(CSRC, f) for f in ("emb_runtime.cu", "emb_inst_f32_f32.cu", "emb_inst_f32_bf16.cu",
                                                        "emb_inst_bf16_f32.cu", "emb_inst_bf16_bf16.cu")],
-                deps=[os.path.join(CSRC, "emb_kernels.cuh"), os.path.join(CSRC, "emb_dispatch.h"), os.path.join(CSRC, "emb_bwd.cuh"),
+                deps=[os.path.join(CSRC, "emb_kernels.cuh"), os.path.join(CSRC, "emb_dispatch.h"), os.path.join(CSRC, "emb_bwd.cuh"), os.path.join(CSRC, "emb_bwd_sort.cuh"),
                       os.path.join(ROOT, "include", "emb.h")],
                 out=os.path.join(PKG, "libemb.so")),
     "synth": dict(srcs=[os.path.join(ROOT, "synth", "csrc", "synth_gen.cu")],

@@ -1,0 +1,376 @@
+// emb_bwd_sort.cuh -- SURVEY row f2, second algorithm ("bwd_algo" = 1): the EMB backward
+// as a transpose of the sparse input (counting sort of the lookups by dW row) followed by
+// a segmented gather-sum, so every distinct dW row receives ONE atomic add per segment of
+// the sorted list instead of one per bag slice.
+//
+// Same definition as emb_bwd.cuh (§V; adjoint of the sum pooling of
+// L91-95):   dW_t[x, :] += sum over bags (t, b), positions j with x_t[j] = x, of dY[b, t, :]
+//
+// Steps (all stream-ordered on the caller's stream; only step 5 reads peers' memory):
+//   1. hist     cnt[g] = number of lookups of global row g (g = rowbase[t] + x), warp-
+//               aggregated atomics (zipf-hot rows repeat inside a warp's 32 lookups)
+//   2. scan     cnt <- exclusive prefix sum (3 kernels: tile sums, scan of the tile sums,
+//               tile scan + offset)
+//   3. scatter  every lookup (t, b, x) writes {dY row code of (b, t), g} at cnt[g]++ ; the
+//               code is (owning DP rank << 28) | (b - s_dst) * T + t_global
+//   4. (memset of cnt before step 1)
+//   5. reduce   persistent warps claim tasks of S consecutive sorted entries, gather each
+//               entry's dY vector (one-sided load from the DP rank's grad slot), sum runs of
+//               equal g in registers and red.add the run into dW_t[x] (two-group software
+//               pipeline of row loads as in the forward); the last CTA releases "done".
+// Order of the fp32 sum inside a run follows the atomic cursor of step 3 (unspecified), so
+// results match the oracle within the order-independent bound and exactly on integer-valued
+// gradients, like the atomic-scatter algorithm.
+#pragma once
+
+#include "emb_bwd.cuh"
+
+namespace emb {
+
+struct SortParams {
+  const int64_t* offsets;      // [T_r*B + 1]
+  const int64_t* indices;
+  const int64_t* rowbase;      // [T_r + 1] global row base of each local table (device)
+  const TableDesc* tables;     // [T_r] (global id)
+  uint32_t* cnt;               // [R] counts -> exclusive starts -> ends
+  uint2* pairs;                // [cap] {dY row code, global row g}
+  uint32_t* bsum;              // [nblk] scan tile sums
+  float* const* dW;            // [T_r] fp32 [M_t][d]
+  const char* gsrc[kMaxG];     // per DP rank: its grad slot of this epoch, [B_dst][T][d] fp32
+  uint32_t* peer_done[kMaxG];  // &done_p[rank] on peer p
+  const uint32_t* my_ready;    // ready_r[G]
+  Ctrl* ctrl;                  // bwork / bdone
+  int64_t bstart[kMaxG + 1];
+  int64_t R, cap, B, timeout_ns;
+  int32_t T, T_r, d, G, rank, lanes, chunk_rows;
+  uint32_t epoch;
+};
+
+constexpr int kScanTile = 4096;    // counters per scan tile (256 threads x 16)
+constexpr int kHistSpan = 1024;    // lookups per warp task in hist
+constexpr int kSortTask = 256;     // sorted entries per warp task in reduce
+
+__device__ __forceinline__ int64_t sort_nnz(const SortParams& p) {
+  return __ldg(p.offsets + (int64_t)p.T_r * p.B);
+}
+
+// local table of position j: the last t with offsets[t*B] <= j (tb in shared memory)
+__device__ __forceinline__ int table_of(const int64_t* tb, int T_r, int64_t j) {
+  int lo = 0, hi = T_r - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (tb[mid] <= j) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+// 1. histogram of lookups per global row
+__global__ void __launch_bounds__(kBlock) emb_bsort_hist_kernel(const __grid_constant__ SortParams p) {
+  extern __shared__ __align__(16) int64_t bs_smem[];
+  int64_t* tb = bs_smem;                    // [T_r + 1] table position bounds
+  int64_t* rb = bs_smem + p.T_r + 1;        // [T_r + 1] row bases
+  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) {
+    tb[i] = __ldg(p.offsets + (int64_t)i * p.B);
+    rb[i] = __ldg(p.rowbase + i);
+  }
+  __syncthreads();
+  const int64_t nnz = tb[p.T_r];
+  if (nnz > p.cap) {                         // workspace too small: skip the step (sticky error)
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr(&p.ctrl->err, 0x4u);
+    return;
+  }
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (kBlock / 32);
+  constexpr int KB = 8;                                   // index loads in flight per lane
+  for (int64_t task = (int64_t)blockIdx.x * (kBlock / 32) + (threadIdx.x >> 5); task * kHistSpan < nnz; task += nw) {
+    const int64_t j0 = task * kHistSpan, j1 = min(nnz, j0 + kHistSpan);
+    int t = table_of(tb, p.T_r, j0 + lane);
+    for (int64_t jb = j0; jb < j1; jb += 32 * KB) {
+      int64_t x[KB];
+#pragma unroll
+      for (int k = 0; k < KB; ++k) {
+        const int64_t j = jb + 32 * k + lane;
+        x[k] = j < j1 ? ld_stream_i64(p.indices + j) : 0;
+      }
+#pragma unroll
+      for (int k = 0; k < KB; ++k) {
+        const int64_t j = jb + 32 * k + lane;
+        const bool valid = j < j1;
+        uint32_t g = 0xffffffffu;
+        if (valid) {
+          while (j >= tb[t + 1]) ++t;
+          g = (uint32_t)(rb[t] + x[k]);
+        }
+        const unsigned same = __match_any_sync(kFull, g);
+        if (valid && (__ffs(same) - 1) == lane) atomicAdd(p.cnt + g, (uint32_t)__popc(same));
+      }
+    }
+  }
+}
+
+// 2a. per-tile sums
+__global__ void __launch_bounds__(kBlock) emb_bsort_scan_sum_kernel(const __grid_constant__ SortParams p) {
+  __shared__ uint32_t red[kBlock / 32];
+  const int64_t base = (int64_t)blockIdx.x * kScanTile;
+  uint32_t s = 0;
+#pragma unroll
+  for (int k = 0; k < kScanTile / kBlock; ++k) {
+    const int64_t i = base + (int64_t)k * kBlock + threadIdx.x;
+    if (i < p.R) s += p.cnt[i];
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    s = threadIdx.x < kBlock / 32 ? red[threadIdx.x] : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+    if (threadIdx.x == 0) p.bsum[blockIdx.x] = s;
+  }
+}
+
+// block-wide exclusive scan of one value per thread (256 threads); returns the block total
+__device__ __forceinline__ uint32_t block_exscan(uint32_t v, uint32_t* sh, uint32_t* total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sh[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t s = lane < kBlock / 32 ? sh[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < kBlock / 32) sh[lane] = s;    // inclusive warp totals
+  }
+  __syncthreads();
+  const uint32_t before = (w > 0 ? sh[w - 1] : 0u) + x - v;
+  *total = sh[kBlock / 32 - 1];
+  __syncthreads();
+  return before;
+}
+
+// 2b. exclusive scan of the tile sums (one CTA, sequential over 256-wide pieces)
+__global__ void __launch_bounds__(kBlock) emb_bsort_scan_top_kernel(uint32_t* bsum, int64_t nblk) {
+  __shared__ uint32_t sh[kBlock / 32];
+  uint32_t carry = 0;
+  for (int64_t b0 = 0; b0 < nblk; b0 += kBlock) {
+    const int64_t i = b0 + threadIdx.x;
+    const uint32_t v = i < nblk ? bsum[i] : 0u;
+    uint32_t tot;
+    const uint32_t ex = block_exscan(v, sh, &tot);
+    if (i < nblk) bsum[i] = carry + ex;
+    carry += tot;
+  }
+}
+
+// 2c. in-place exclusive scan of each tile plus its offset: 16 coalesced rounds of 256
+__global__ void __launch_bounds__(kBlock) emb_bsort_scan_apply_kernel(const __grid_constant__ SortParams p) {
+  __shared__ uint32_t sh[kBlock / 32];
+  const int64_t base = (int64_t)blockIdx.x * kScanTile + threadIdx.x;
+  uint32_t v[kScanTile / kBlock];
+#pragma unroll
+  for (int k = 0; k < kScanTile / kBlock; ++k) v[k] = (base + k * kBlock < p.R) ? p.cnt[base + k * kBlock] : 0u;
+  uint32_t carry = p.bsum[blockIdx.x];
+#pragma unroll
+  for (int k = 0; k < kScanTile / kBlock; ++k) {
+    uint32_t tot;
+    const uint32_t ex = block_exscan(v[k], sh, &tot);
+    if (base + k * kBlock < p.R) p.cnt[base + k * kBlock] = carry + ex;
+    carry += tot;
+  }
+}
+
+// 3. scatter every lookup to its row's segment: warp per chunk of consecutive bags of one
+// table; each lane finds its position's bag in the chunk's offsets (shared memory)
+__global__ void __launch_bounds__(kBlock) emb_bsort_scatter_kernel(const __grid_constant__ SortParams p) {
+  __shared__ int64_t ofs[kBlock / 32][33];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t B = p.B, nbags = (int64_t)p.T_r * B;
+  if (nbags == 0) return;
+  const int64_t nnz = sort_nnz(p);
+  if (nnz > p.cap) return;
+  const int64_t cb64 = nnz > 0 ? ((int64_t)p.chunk_rows * nbags + nnz - 1) / nnz : 31;
+  const int cb = (int)(cb64 < 1 ? 1 : (cb64 > 31 ? 31 : cb64));
+  const int64_t cpt = (B + cb - 1) / cb, nchunks = cpt * p.T_r;
+  const int64_t nw = (int64_t)gridDim.x * (kBlock / 32);
+  for (int64_t c = (int64_t)blockIdx.x * (kBlock / 32) + w; c < nchunks; c += nw) {
+    const int t_l = (int)(c / cpt);
+    const int64_t b0 = (c % cpt) * cb;
+    const int nb = (int)min((int64_t)cb, B - b0);
+    if (lane <= nb) ofs[w][lane] = ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane);
+    __syncwarp();
+    const int64_t pos0 = ofs[w][0], pos1 = ofs[w][nb];
+    const int64_t rb = __ldg(p.rowbase + t_l);
+    const int64_t tglob = __ldg(&p.tables[t_l].tglob);
+    constexpr int KB = 4;                                 // batches of 32 lookups in flight
+    for (int64_t jb = pos0; jb < pos1; jb += 32 * KB) {
+      int64_t x[KB];
+#pragma unroll
+      for (int k = 0; k < KB; ++k) {
+        const int64_t j = jb + 32 * k + lane;
+        x[k] = j < pos1 ? ld_stream_i64(p.indices + j) : 0;
+      }
+      uint32_t g[KB], code[KB], at[KB];
+      unsigned same[KB];
+#pragma unroll
+      for (int k = 0; k < KB; ++k) {
+        const int64_t j = jb + 32 * k + lane;
+        const bool valid = j < pos1;
+        g[k] = 0xffffffffu;
+        code[k] = 0;
+        if (valid) {
+          int lo = 0, hi = nb - 1;                  // last bag with start <= j
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (ofs[w][mid] <= j) lo = mid;
+            else hi = mid - 1;
+          }
+          const int64_t b = b0 + lo;
+          int dst = 0;
+          while (b >= p.bstart[dst + 1]) ++dst;
+          code[k] = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
+          g[k] = (uint32_t)(rb + x[k]);
+        }
+        same[k] = __match_any_sync(kFull, g[k]);
+        at[k] = 0;
+        if (valid && (__ffs(same[k]) - 1) == lane) at[k] = atomicAdd(p.cnt + g[k], (uint32_t)__popc(same[k]));
+      }
+#pragma unroll
+      for (int k = 0; k < KB; ++k) {
+        const int64_t j = jb + 32 * k + lane;
+        const int leader = __ffs(same[k]) - 1;
+        const uint32_t a = __shfl_sync(kFull, at[k], leader) + (uint32_t)__popc(same[k] & ((1u << lane) - 1u));
+        if (j < pos1) p.pairs[a] = make_uint2(code[k], g[k]);
+      }
+    }
+    __syncwarp();
+  }
+}
+
+// 5. segmented gather-sum of the sorted entries + one red.add per run of equal rows
+template <int VB, int NV>
+__global__ void __launch_bounds__(kBlock) emb_bsort_reduce_kernel(const __grid_constant__ SortParams p) {
+  constexpr int W = VB / 4;
+  constexpr int UR = 4;                                   // rows per pipeline group
+  extern __shared__ __align__(16) int64_t bs_smem[];
+  int64_t* rb = bs_smem;                                  // [T_r + 1] row bases
+  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) rb[i] = __ldg(p.rowbase + i);
+  const int lane = threadIdx.x & 31;
+  const bool active = lane < p.lanes;
+  const int64_t rowbytes = (int64_t)p.d * 4;
+  if (threadIdx.x == 0 && p.G > 1) wait_flags_geq(p.my_ready, p.G, p.rank, p.epoch, p.timeout_ns, &p.ctrl->err);
+  __syncthreads();
+  const int64_t nnz = sort_nnz(p);
+  if (nnz <= p.cap) {
+    const int64_t ntask = (nnz + kSortTask - 1) / kSortTask;
+    unsigned c_next = 0;
+    if (lane == 0) c_next = atomicAdd(&p.ctrl->bwork, 1u);
+    for (;;) {
+      const unsigned c = __shfl_sync(kFull, c_next, 0);
+      if ((int64_t)c >= ntask) break;
+      if (lane == 0) c_next = atomicAdd(&p.ctrl->bwork, 1u);
+      const int64_t e0 = (int64_t)c * kSortTask, e1 = min(nnz, e0 + kSortTask);
+      const int n = (int)(e1 - e0);
+      // this task's entries, one per lane per batch of 32
+      uint2 ent = lane < n ? p.pairs[e0 + lane] : make_uint2(0u, 0xffffffffu);
+      uint32_t cur = __shfl_sync(kFull, ent.y, 0);        // row of the current run
+      int t = 0;
+      {
+        int lo = 0, hi = p.T_r - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (rb[mid] <= (int64_t)cur) lo = mid;
+          else hi = mid - 1;
+        }
+        t = lo;
+      }
+      float acc[NV * W];
+#pragma unroll
+      for (int i = 0; i < NV * W; ++i) acc[i] = 0.0f;
+      auto emit = [&]() {                                 // run of row `cur` -> dW_t[x]
+        while ((int64_t)cur >= rb[t + 1]) ++t;
+        if (active) {
+          float* dwt = reinterpret_cast<float*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t)));
+          char* rp = reinterpret_cast<char*>(dwt) + ((int64_t)cur - rb[t]) * rowbytes + lane * VB;
+#pragma unroll
+          for (int v = 0; v < NV; ++v) {
+            uint32_t u[W];
+#pragma unroll
+            for (int i = 0; i < W; ++i) u[i] = __float_as_uint(acc[v * W + i]);
+            red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), u);
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < NV * W; ++i) acc[i] = 0.0f;
+      };
+      auto gaddr = [&](uint32_t code) -> const char* {
+        return p.gsrc[code >> 28] + (int64_t)(code & 0x0fffffffu) * rowbytes + lane * VB;
+      };
+      uint32_t bufA[UR][NV][W], bufB[UR][NV][W];
+      uint32_t gA[UR], gB[UR];
+      auto issue = [&](uint32_t (&buf)[UR][NV][W], uint32_t (&gg)[UR], const uint2& e, int j0, int jn) {
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+          const int j = j0 + u;
+          const uint32_t code = __shfl_sync(kFull, e.x, j & 31);
+          gg[u] = __shfl_sync(kFull, e.y, j & 31);
+          if (j < jn && active) {
+            const char* a = gaddr(code);
+#pragma unroll
+            for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, buf[u][v]);
+          }
+        }
+      };
+      auto consume = [&](const uint32_t (&buf)[UR][NV][W], const uint32_t (&gg)[UR], int j0, int jn) {
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+          if (j0 + u < jn) {
+            if (gg[u] != cur) {
+              emit();
+              cur = gg[u];
+            }
+#pragma unroll
+            for (int v = 0; v < NV; ++v)
+#pragma unroll
+              for (int i = 0; i < W; ++i) acc[v * W + i] += __uint_as_float(buf[u][v][i]);
+          }
+        }
+      };
+      for (int base = 0; base < n; base += 32) {
+        const int jn = min(32, n - base);
+        if (base > 0) ent = (base + lane < n) ? p.pairs[e0 + base + lane] : make_uint2(0u, 0xffffffffu);
+        issue(bufA, gA, ent, 0, jn);
+#pragma unroll 1
+        for (int j = 0; j < jn; j += 2 * UR) {
+          issue(bufB, gB, ent, j + UR, jn);
+          consume(bufA, gA, j, jn);
+          if (j + 2 * UR < jn) issue(bufA, gA, ent, j + 2 * UR, jn);
+          consume(bufB, gB, j + UR, jn);
+        }
+      }
+      emit();                                             // the task's last run
+    }
+  }
+  // completion: every CTA's reads of peer slots are done before the last CTA tells the
+  // peers their slots may be refilled
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  fence_acq_rel_sys();
+  const unsigned prev = atomicAdd(&p.ctrl->bdone, 1u);
+  if (prev != gridDim.x - 1) return;
+  fence_acq_rel_sys();
+  p.ctrl->bdone = 0;
+  p.ctrl->bwork = 0;
+  for (int q = 1; q < p.G; ++q) st_release_sys(p.peer_done[(p.rank + q) % p.G], p.epoch);
+}
+
+}  // namespace emb

@@ -26,6 +26,7 @@
 #include "emb_kernels.cuh"
 #include "emb_dispatch.h"
 #include "emb_bwd.cuh"
+#include "emb_bwd_sort.cuh"
 
 using namespace emb;
 
@@ -125,6 +126,12 @@ struct emb_ctx {
   int bwd_cache = 16;              // per-warp dW row cache slots (0 off; 8 / 16 / 32; needs bwd_v2)
   int bwd_chunk_rows = 0;          // backward chunk target rows (0: chunk_rows)
   int bwd_group = 4;               // tables interleaved at a time in the backward (0: all T_r)
+  int bwd_algo = 0;                // 0: atomic scatter per bag slice; 1: counting sort + segmented sum
+  int64_t bs_cap = 0, bs_R = 0, bs_nblk = 0;   // bwd_algo 1 workspace
+  int64_t* d_rowbase = nullptr;
+  uint32_t* d_bcnt = nullptr;
+  uint32_t* d_bsum = nullptr;
+  uint2* d_pairs = nullptr;
   int fwd_interleave = 0;
   int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
   int tail_div = 4;                // guided tail of the forward's chunk schedule
@@ -493,6 +500,15 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2, true>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4, true>);
+    cudaFuncGetAttributes(&a, emb_bsort_hist_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_scan_sum_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_scan_top_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_scan_apply_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_scatter_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 4>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 8>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 16>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 32>);
@@ -858,6 +874,85 @@ emb_status_t emb_backward_grad_ready(emb_ctx_t* c, void* stream) {
   return EMB_OK;
 }
 
+// f2, bwd_algo 1 (emb_bwd_sort.cuh): counting sort of the lookups by dW row, then a
+// segmented gather-sum with one red.add per run of equal rows
+static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int64_t* offsets, const int64_t* indices,
+                                    cudaStream_t s) {
+  if (!c->d_rowbase) {                                  // workspace sized by the local rows
+    std::vector<int64_t> rb(c->T_r + 1, 0);
+    for (int i = 0; i < c->T_r; ++i) rb[i + 1] = rb[i] + c->rows[c->local[i]];
+    if (rb[c->T_r] >= 0xffffffffll) FAIL(c, EMB_ERR_ARG, "bwd_algo 1: more than 2^32-2 local rows");
+    const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+    for (int g = 0; g < c->G; ++g)
+      if ((c->bstart[g + 1] - c->bstart[g]) * (int64_t)c->T >= (1ll << 28))
+        FAIL(c, EMB_ERR_ARG, "bwd_algo 1: B_r * T must be < 2^28 (B_r = %lld)", (long long)Br);
+    c->bs_R = rb[c->T_r];
+    c->bs_nblk = (c->bs_R + kScanTile - 1) / kScanTile;
+    CK(c, cudaMalloc(&c->d_rowbase, rb.size() * sizeof(int64_t)));
+    CK(c, cudaMemcpy(c->d_rowbase, rb.data(), rb.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+    CK(c, cudaMalloc(&c->d_bcnt, std::max<int64_t>(c->bs_R, 1) * sizeof(uint32_t)));
+    CK(c, cudaMalloc(&c->d_bsum, std::max<int64_t>(c->bs_nblk, 1) * sizeof(uint32_t)));
+  }
+  if (!c->d_pairs) {                                    // entry list: sized from the first CSR
+    if (c->bs_cap <= 0) {                               // (one host sync, first call only)
+      int64_t nnz = 0;
+      CK(c, cudaMemcpyAsync(&nnz, offsets + (int64_t)c->T_r * c->B, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+      CK(c, cudaStreamSynchronize(s));
+      c->bs_cap = std::min<int64_t>(nnz + nnz / 4 + 4096, 0xffffffffll);
+    }
+    CK(c, cudaMalloc(&c->d_pairs, (size_t)c->bs_cap * sizeof(uint2)));
+  }
+  SortParams q;
+  memset(&q, 0, sizeof(q));
+  q.offsets = offsets;
+  q.indices = indices;
+  q.rowbase = c->d_rowbase;
+  q.tables = c->d_tables;
+  q.cnt = c->d_bcnt;
+  q.pairs = c->d_pairs;
+  q.bsum = c->d_bsum;
+  q.dW = bp.dW;
+  for (int g = 0; g < kMaxG; ++g) {
+    q.gsrc[g] = bp.gsrc[g];
+    q.peer_done[g] = bp.peer_done[g];
+  }
+  for (int g = 0; g <= kMaxG; ++g) q.bstart[g] = bp.bstart[g];
+  q.my_ready = bp.my_ready;
+  q.ctrl = c->ctrl;
+  q.R = c->bs_R;
+  q.cap = c->bs_cap;
+  q.B = c->B;
+  q.timeout_ns = c->timeout_ns;
+  q.T = c->T;
+  q.T_r = c->T_r;
+  q.d = c->d;
+  q.G = c->G;
+  q.rank = c->rank;
+  q.lanes = c->blanes;
+  q.chunk_rows = c->chunk_rows;
+  q.epoch = bp.epoch;
+  const size_t tsm = (size_t)(c->T_r + 1) * 2 * sizeof(int64_t);
+  const int grid = c->num_sms * 8;
+  CK(c, cudaMemsetAsync(c->d_bcnt, 0, (size_t)c->bs_R * sizeof(uint32_t), s));
+  emb_bsort_hist_kernel<<<grid, kBlock, tsm, s>>>(q);
+  if (c->bs_nblk > 0) {
+    emb_bsort_scan_sum_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
+    emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_bsum, c->bs_nblk);
+    emb_bsort_scan_apply_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
+  }
+  emb_bsort_scatter_kernel<<<grid, kBlock, 0, s>>>(q);
+  void (*k)(SortParams) = nullptr;
+  if (c->bvb == 8) k = emb_bsort_reduce_kernel<8, 1>;
+  else if (c->bnv == 2) k = emb_bsort_reduce_kernel<16, 2>;
+  else if (c->bnv == 4) k = emb_bsort_reduce_kernel<16, 4>;
+  else k = emb_bsort_reduce_kernel<16, 1>;
+  int per_sm = 0;
+  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, tsm / 2));
+  k<<<c->num_sms * std::max(per_sm, 1), kBlock, tsm / 2, s>>>(q);
+  CK(c, cudaGetLastError());
+  return EMB_OK;
+}
+
 emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, void* const* dW,
                           uint32_t flags, void* stream) {
   (void)flags;
@@ -880,6 +975,8 @@ emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* i
   c->bwd_ready_pending = false;
   BwdParams p;
   fill_bwd_params(c, &p);
+  if (c->bwd_algo == 1 && c->T_r > 0 && c->T_r <= 2048)
+    return backward_sorted(c, p, offsets, indices, s);
   p.offsets = offsets;
   p.indices = indices;
   void (*k)(BwdParams) = nullptr;
@@ -954,6 +1051,10 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->s_in) cudaStreamDestroy(c->s_in);
   if (c->trace) cudaFree(c->trace);
   if (c->d_dW) cudaFree(c->d_dW);
+  if (c->d_rowbase) cudaFree(c->d_rowbase);
+  if (c->d_bcnt) cudaFree(c->d_bcnt);
+  if (c->d_bsum) cudaFree(c->d_bsum);
+  if (c->d_pairs) cudaFree(c->d_pairs);
   if (c->s_out) cudaStreamDestroy(c->s_out);
   delete c;
   return st;
@@ -1028,6 +1129,12 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "bwd_v2")) c->bwd_v2 = v ? 1 : 0;
+  else if (!strcmp(key, "bwd_algo")) { if (v != 0 && v != 1) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0 or 1"); c->bwd_algo = (int)v; }
+  else if (!strcmp(key, "bwd_max_nnz")) {
+    if (v < 0 || v >= (1ll << 32)) FAIL(c, EMB_ERR_ARG, "bwd_max_nnz not in [0, 2^32)");
+    if (c->d_pairs) { cudaFree(c->d_pairs); c->d_pairs = nullptr; }
+    c->bs_cap = v;
+  }
   else if (!strcmp(key, "bwd_cache")) {
     if (v != 0 && v != 8 && v != 16 && v != 32) FAIL(c, EMB_ERR_ARG, "bwd_cache must be 0, 8, 16 or 32");
     c->bwd_cache = (int)v;

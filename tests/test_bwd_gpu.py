@@ -107,7 +107,7 @@ def test_bwd_placement_invariance():
                                   {"bwd_group": 7}, {"bwd_group": 1}, {"bwd_v2": 1}, {"bwd_v2": 1, "bwd_group": 3},
                                   {"bwd_v2": 1, "bwd_interleave": 0}, {"bwd_v2": 1, "bwd_cache": 8},
                                   {"bwd_v2": 1, "bwd_cache": 16, "bwd_chunk_rows": 1024},
-                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}])
+                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}, {"bwd_algo": 1}])
 def test_bwd_chunk_orders_integer_exact(opts):
     """every chunk order (table-major, groups of g tables incl. a ragged last group, all
     tables interleaved) visits every bag exactly once: exact on integer gradients"""
@@ -119,11 +119,12 @@ def test_bwd_chunk_orders_integer_exact(opts):
         assert np.array_equal(got[t].astype(np.float64), ref[t]), t
 
 
-@pytest.mark.parametrize("dim,cache", [(16, 8), (64, 16), (128, 32), (256, 8)])
+@pytest.mark.parametrize("dim,cache", [(16, 8), (64, 16), (128, 32), (256, 8), (16, -1), (64, -1), (128, -1),
+                                       (256, -1), (512, -1)])
 def test_bwd_row_cache_exact_and_float_bound(dim, cache):
     """f2 per-warp dW row cache (bwd_cache): integer gradients exact, float gradients within
     the order-independent summation bound (cached rows are summed in shared memory first)"""
-    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512}
+    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512} if cache > 0 else {"bwd_algo": 1}
     w = synth.make_workload("tiny", G=2, pmin=0, pmax=60, B=150, T=3, dim=dim, rows=200, dist="zipf")
     got, offs, idxs = _run_bwd(w, _dY(w, 21, integer=True), 22, opts=opts)
     ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, _dY(w, 21, integer=True), w.B, w.G)
@@ -136,3 +137,35 @@ def test_bwd_row_cache_exact_and_float_bound(dim, cache):
         n = 2 * cnt[t][:, None]
         err = np.abs(got[t].astype(np.float64) - 2 * ref[t])
         assert np.all(err <= n * 2.0 ** -24 * 2 * S[t] + 1e-30), t
+
+
+@pytest.mark.parametrize("G,dist", [(1, "zipf"), (2, "uniform"), (3, "zipf")])
+def test_bwd_sorted_algo_integer_exact_multi_epoch(G, dist):
+    """bwd_algo 1 (counting sort + segmented sum): exact on integer gradients over 3 epochs
+    (workspace reuse, counters re-zeroed), incl. empty bags and G > 1 one-sided dY loads"""
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=70, B=131, T=5, dim=128, rows=400, dist=dist)
+    dY = _dY(w, 31, integer=True)
+    got, offs, idxs = _run_bwd(w, dY, 32, epochs=3, opts={"bwd_algo": 1})
+    ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    for t in range(w.T):
+        assert np.array_equal(got[t].astype(np.float64), 3 * ref[t]), t
+
+
+def test_bwd_sorted_capacity_error():
+    """a CSR with more lookups than the preset workspace sets EMB_DEVERR_CAPACITY (0x4)"""
+    w = synth.make_workload("tiny", G=1, pmin=1, pmax=20, B=64, T=2, dim=32, rows=100)
+    tabs = H.np_tables(w)
+    offs, idxs = H.np_csrs(w, 5)
+    L = PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, [torch.from_numpy(tabs[int(w.phys[t])]).to(DEV) for t in range(w.T)],
+                      w.B, backward=True)
+    try:
+        E.emb_set_option(L.ctx, "bwd_algo", 1)
+        E.emb_set_option(L.ctx, "bwd_max_nnz", 10)
+        dW = [torch.zeros((int(w.rows[t]), w.dim), device=DEV) for t in range(w.T)]
+        g = L.grad_slot()
+        g.zero_()
+        L.backward(torch.from_numpy(offs[0]).to(DEV), torch.from_numpy(idxs[0]).to(DEV), dW)
+        torch.cuda.synchronize()
+        assert L.device_error(clear=True) & 0x4
+    finally:
+        L.close()
