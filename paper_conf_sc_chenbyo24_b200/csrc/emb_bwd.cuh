@@ -246,10 +246,15 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
                     const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
                     const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
                     const uint32_t h = HC == 1 ? 0u : (xl * 2654435761u) >> (32 - kLogHC);
-                    uint32_t tg;
-                    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * h) : "memory");
+                    // lane 0 alone reads and claims the tag (no cross-lane access to it); the
+                    // shuffle hands its decision to the warp
+                    uint32_t tg = 0;
+                    if (lane == 0) {
+                      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * h) : "memory");
+                      if (tg == kEmpty) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * h), "r"(xl) : "memory");
+                    }
+                    tg = __shfl_sync(kFull, tg, 0);
                     const bool hit = tg == xl, claim = tg == kEmpty;
-                    if (claim) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * h), "r"(xl) : "memory");
                     if (active) {
 #pragma unroll
                       for (int v = 0; v < NV; ++v) {

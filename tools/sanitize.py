@@ -1,6 +1,6 @@
 """Small end-to-end run for compute-sanitizer (memcheck / racecheck / synccheck):
 forward at G=1 and simulated G=2 (fused kernel, flags, unpack), pipelined host path and
-backward.  Usage: compute-sanitizer --tool memcheck python tools/sanitize.py"""
+backward (both algorithms).  Usage: compute-sanitizer --tool memcheck python tools/sanitize.py"""
 import os
 import sys
 
@@ -45,6 +45,16 @@ for G in (1, 2):
         b = layers[r].forward_baseline(ins[r][0], ins[r][1]) if G == 1 else None
     dW = [[torch.zeros((int(w.rows[t]), w.dim), device=dev) for t in w.local_tables(r)] for r in range(G)]
     for r in range(G):
+        with torch.cuda.stream(streams[r]):
+            layers[r].grad_slot(streams[r]).fill_(1.0)
+        layers[r].grad_ready(streams[r])
+    torch.cuda.synchronize()
+    for r in range(G):
+        layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
+    torch.cuda.synchronize()
+    # second backward algorithm (counting sort + segmented sum), same slots and flags
+    for r in range(G):
+        E.emb_set_option(layers[r].ctx, "bwd_algo", 1)
         with torch.cuda.stream(streams[r]):
             layers[r].grad_slot(streams[r]).fill_(1.0)
         layers[r].grad_ready(streams[r])
