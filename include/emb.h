@@ -192,7 +192,8 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * 10000 or env EMB_TIMEOUT_MS), "unroll" (row pipeline: 0 = auto (default), 2 or 4 = rows per group of the
  * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
  * flight per warp in a cp.async shared-memory ring), "minblocks" (CTAs of 256 per
- * SM the register budget is sized for: 0 = auto (4 for one vector per lane, else 1), 1, 4, 6).
+ * SM the register budget is sized for: 0 = auto (5 for fp32 rows of one 16-B vector per lane,
+ * 4 for other one-vector-per-lane tiles, else 1), 1, 4, 5, 6).
  * "tma_store" (f4, PAPER.md L386 aggregated stores: 1 = pooled vectors are staged per
  * warp in shared memory and shipped 4 at a time to 4 arbitrary output rows with one TMA
  * scatter4; needs full-warp rows with one vector per lane and d <= 256),

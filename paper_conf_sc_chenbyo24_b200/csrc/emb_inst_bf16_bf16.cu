@@ -25,6 +25,7 @@ KernelFn pick_u(int unroll, int mb, bool full, bool sidx, bool shard, bool tmast
       return sidx ? emb_fwd_kernel<VB, NV, WT, OT, 8, false, 2, true, true> : emb_fwd_kernel<VB, NV, WT, OT, 8, false, 2, true, false>;
     if (sidx && unroll == 4 && mb == 4) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 4, true, true>;
     if (sidx && unroll == 4 && mb == 5) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 5, true, true>;  // 40 warps/SM
+    if (sidx && unroll == 4 && mb == 6) return emb_fwd_kernel<VB, NV, WT, OT, 4, false, 6, true, true>;  // 48 warps/SM
     if (sidx && unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, false, 6, true, true>;
   }
   if (unroll == 2) return emb_fwd_kernel<VB, NV, WT, OT, 2, CHECK, 6, true>;

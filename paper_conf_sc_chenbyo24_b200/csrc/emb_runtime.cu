@@ -164,8 +164,14 @@ struct emb_ctx {
 
 static size_t esize(emb_dtype_t t) { return t == EMB_F32 ? 4 : 2; }
 // register budget per tile: one vector per lane fits 64 registers (4 CTAs of 256 per SM,
-// no spills for any dtype pair); wider rows keep the unconstrained build
-static int eff_minblocks(const emb_ctx* c) { return c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1); }
+// no spills for any dtype pair); fp32 rows of 16-B lanes take 48 registers (5 CTAs, 40
+// warps/SM: zipf weak 0.70 -> 0.67 ms, strong 6.66 -> 6.39 ms; uniform +0.4 %; bf16 rows
+// spill at 48 and stay at 4); wider rows keep the unconstrained build
+static int eff_minblocks(const emb_ctx* c) {
+  if (c->minblocks) return c->minblocks;
+  if (c->nv != 1) return 1;
+  return (c->vb == 16 && c->wdt == EMB_F32) ? 5 : 4;
+}
 // rows per pipeline group: 4 rows for both 8- and 16-byte lane vectors (measured best)
 static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4); }
 // a row exactly covers the warp's 32 lane vectors (lets the row stride be a constant)
@@ -175,9 +181,9 @@ static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d 
 // per lane, no bounds check, no row shards, direct stores, 4-row groups (or 2 with 8-B lanes)
 static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
   const int u = c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4);
-  const int mb = c->minblocks ? c->minblocks : (c->nv == 1 ? 4 : 1);
+  const int mb = eff_minblocks(c);
   return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
-         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && (mb == 4 || mb == 5)) || u == 2 || u == 3);
+         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && (mb == 4 || mb == 5 || mb == 6)) || u == 2 || u == 3);
 }
 // dual-stream kernel (emb_fwd_ds_kernel): 256-B rows, default options, no bounds check,
 // no row shards, direct stores
