@@ -256,6 +256,181 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_scatter_kernel(const __grid_
   }
 }
 
+// ---------------------------------------------------------------------------- bwd_algo 2
+// Same sort, but the histogram and the scatter first aggregate a CTA's span of lookups in
+// a shared-memory hash table (open addressing, kHashSlots keys + counts): a zipf-hot row
+// then costs ONE global atomic per span instead of one per 32 lookups (the same-address
+// atomics on hot counters are what serialize bwd_algo 1).  Keys that find no free slot
+// within kHashProbe probes go straight to the global counter.
+constexpr int kHashSlots = 8192;   // smem: keys + counts (+ bases in scatter) per CTA
+constexpr int kHashProbe = 8;
+constexpr int kHashSpan = 4096;    // lookups per CTA task (load factor <= 1/2)
+constexpr uint32_t kHashEmpty = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t hslot(uint32_t k) { return (k * 2654435761u) >> (32 - 13); }
+
+// insert `c` occurrences of key k; returns false if no slot was found (caller goes global)
+__device__ __forceinline__ bool hash_add(uint32_t* hk, uint32_t* hc, uint32_t k, uint32_t c) {
+  uint32_t h = hslot(k);
+#pragma unroll 1
+  for (int i = 0; i < kHashProbe; ++i) {
+    const uint32_t old = atomicCAS(hk + h, kHashEmpty, k);
+    if (old == kHashEmpty || old == k) {
+      atomicAdd(hc + h, c);
+      return true;
+    }
+    h = (h + 1) & (kHashSlots - 1);
+  }
+  return false;
+}
+
+__device__ __forceinline__ int hash_find(const uint32_t* hk, uint32_t k) {
+  uint32_t h = hslot(k);
+#pragma unroll 1
+  for (int i = 0; i < kHashProbe; ++i) {
+    const uint32_t v = hk[h];
+    if (v == k) return (int)h;
+    if (v == kHashEmpty) return -1;
+    h = (h + 1) & (kHashSlots - 1);
+  }
+  return -1;
+}
+
+// 1'. histogram with per-CTA aggregation over spans of kHashSpan consecutive lookups
+__global__ void __launch_bounds__(kBlock) emb_bsort_hist2_kernel(const __grid_constant__ SortParams p) {
+  extern __shared__ __align__(16) uint32_t hs_smem[];
+  uint32_t* hk = hs_smem;
+  uint32_t* hc = hs_smem + kHashSlots;
+  int64_t* tb = reinterpret_cast<int64_t*>(hs_smem + 2 * kHashSlots);
+  int64_t* rb = tb + p.T_r + 1;
+  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) {
+    tb[i] = __ldg(p.offsets + (int64_t)i * p.B);
+    rb[i] = __ldg(p.rowbase + i);
+  }
+  for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
+    hk[i] = kHashEmpty;
+    hc[i] = 0;
+  }
+  __syncthreads();
+  const int64_t nnz = tb[p.T_r];
+  if (nnz > p.cap) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr(&p.ctrl->err, 0x4u);
+    return;
+  }
+  const int lane = threadIdx.x & 31;
+  for (int64_t task = blockIdx.x; task * kHashSpan < nnz; task += gridDim.x) {
+    const int64_t j0 = task * kHashSpan, j1 = min(nnz, j0 + kHashSpan);
+    constexpr int KB = kHashSpan / kBlock;               // 16 lookups per thread
+    int64_t x[KB];
+#pragma unroll
+    for (int k = 0; k < KB; ++k) {
+      const int64_t j = j0 + (int64_t)k * kBlock + threadIdx.x;
+      x[k] = j < j1 ? ld_stream_i64(p.indices + j) : 0;
+    }
+    int t = table_of(tb, p.T_r, j0 + threadIdx.x);
+#pragma unroll
+    for (int k = 0; k < KB; ++k) {
+      const int64_t j = j0 + (int64_t)k * kBlock + threadIdx.x;
+      const bool valid = j < j1;
+      uint32_t g = kHashEmpty;
+      if (valid) {
+        while (j >= tb[t + 1]) ++t;
+        g = (uint32_t)(rb[t] + x[k]);
+      }
+      const unsigned same = __match_any_sync(kFull, g);
+      if (valid && (__ffs(same) - 1) == lane && !hash_add(hk, hc, g, (uint32_t)__popc(same)))
+        atomicAdd(p.cnt + g, (uint32_t)__popc(same));
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {   // flush + clear
+      const uint32_t k = hk[i];
+      if (k != kHashEmpty) {
+        atomicAdd(p.cnt + k, hc[i]);
+        hk[i] = kHashEmpty;
+        hc[i] = 0;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// 3'. scatter with per-CTA aggregation: CTA task = a chunk of consecutive bags of one table
+// (<= 1024 bags, ~kHashSpan lookups).  Pass 1 counts the chunk's keys in the hash table,
+// then one returning global atomic per distinct key reserves its run, pass 2 hands out
+// positions inside the runs with shared-memory atomics.
+__global__ void __launch_bounds__(kBlock) emb_bsort_scatter2_kernel(const __grid_constant__ SortParams p) {
+  constexpr int kMaxCB = 1024;
+  extern __shared__ __align__(16) uint32_t hs_smem[];
+  uint32_t* hk = hs_smem;
+  uint32_t* hc = hs_smem + kHashSlots;                    // counts, then local cursors
+  uint32_t* hb = hs_smem + 2 * kHashSlots;                // reserved global base per key
+  int64_t* ofs = reinterpret_cast<int64_t*>(hs_smem + 3 * kHashSlots);   // [kMaxCB + 1]
+  const int64_t B = p.B, nbags = (int64_t)p.T_r * B;
+  if (nbags == 0) return;
+  const int64_t nnz = sort_nnz(p);
+  if (nnz > p.cap) return;
+  for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
+    hk[i] = kHashEmpty;
+    hc[i] = 0;
+  }
+  const int64_t cb64 = nnz > 0 ? ((int64_t)kHashSpan * nbags + nnz - 1) / nnz : kMaxCB;
+  const int cb = (int)(cb64 < 1 ? 1 : (cb64 > kMaxCB ? kMaxCB : cb64));
+  const int64_t cpt = (B + cb - 1) / cb, nchunks = cpt * p.T_r;
+  __syncthreads();
+  for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
+    const int t_l = (int)(c / cpt);
+    const int64_t b0 = (c % cpt) * cb;
+    const int nb = (int)min((int64_t)cb, B - b0);
+    for (int i = threadIdx.x; i <= nb; i += blockDim.x) ofs[i] = ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + i);
+    __syncthreads();
+    const int64_t pos0 = ofs[0], pos1 = ofs[nb];
+    const int64_t rb = __ldg(p.rowbase + t_l);
+    const int64_t tglob = __ldg(&p.tables[t_l].tglob);
+    // pass 1: counts
+    for (int64_t j = pos0 + threadIdx.x; j - threadIdx.x < pos1; j += kBlock) {
+      const bool valid = j < pos1;
+      const uint32_t g = valid ? (uint32_t)(rb + ld_stream_i64(p.indices + j)) : kHashEmpty;
+      const unsigned same = __match_any_sync(kFull, g);
+      if (valid && (__ffs(same) - 1) == (int)(threadIdx.x & 31)) hash_add(hk, hc, g, (uint32_t)__popc(same));
+    }
+    __syncthreads();
+    // reserve each key's run: one returning global atomic per distinct key
+    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
+      const uint32_t k = hk[i];
+      if (k != kHashEmpty) {
+        hb[i] = atomicAdd(p.cnt + k, hc[i]);
+        hc[i] = 0;
+      }
+    }
+    __syncthreads();
+    // pass 2: positions
+    for (int64_t j = pos0 + threadIdx.x; j - threadIdx.x < pos1; j += kBlock) {
+      if (j < pos1) {
+        const uint32_t g = (uint32_t)(rb + ld_stream_i64(p.indices + j));
+        int lo = 0, hi = nb - 1;                          // last bag with start <= j
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (ofs[mid] <= j) lo = mid;
+          else hi = mid - 1;
+        }
+        const int64_t b = b0 + lo;
+        int dst = 0;
+        while (b >= p.bstart[dst + 1]) ++dst;
+        const uint32_t code = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
+        const int h = hash_find(hk, g);
+        const uint32_t at = h >= 0 ? hb[h] + atomicAdd(hc + h, 1u) : atomicAdd(p.cnt + g, 1u);
+        p.pairs[at] = make_uint2(code, g);
+      }
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
+      hk[i] = kHashEmpty;
+      hc[i] = 0;
+    }
+    __syncthreads();
+  }
+}
+
 // 5. segmented gather-sum of the sorted entries + one red.add per run of equal rows
 template <int VB, int NV>
 __global__ void __launch_bounds__(kBlock) emb_bsort_reduce_kernel(const __grid_constant__ SortParams p) {

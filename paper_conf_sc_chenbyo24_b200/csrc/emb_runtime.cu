@@ -511,6 +511,8 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bsort_scan_top_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scan_apply_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scatter_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_hist2_kernel);
+    cudaFuncGetAttributes(&a, emb_bsort_scatter2_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2>);
@@ -940,13 +942,23 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   const size_t tsm = (size_t)(c->T_r + 1) * 2 * sizeof(int64_t);
   const int grid = c->num_sms * 8;
   CK(c, cudaMemsetAsync(c->d_bcnt, 0, (size_t)c->bs_R * sizeof(uint32_t), s));
-  emb_bsort_hist_kernel<<<grid, kBlock, tsm, s>>>(q);
+  const bool agg = c->bwd_algo == 2;                   // CTA-level shared-memory aggregation
+  const size_t hsm = (size_t)2 * kHashSlots * sizeof(uint32_t) + tsm;
+  const size_t ssm = (size_t)3 * kHashSlots * sizeof(uint32_t) + 1025 * sizeof(int64_t);
+  if (agg) {
+    CK(c, cudaFuncSetAttribute(emb_bsort_hist2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm));
+    CK(c, cudaFuncSetAttribute(emb_bsort_scatter2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm));
+    emb_bsort_hist2_kernel<<<c->num_sms * 3, kBlock, hsm, s>>>(q);
+  } else {
+    emb_bsort_hist_kernel<<<grid, kBlock, tsm, s>>>(q);
+  }
   if (c->bs_nblk > 0) {
     emb_bsort_scan_sum_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
     emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_bsum, c->bs_nblk);
     emb_bsort_scan_apply_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
   }
-  emb_bsort_scatter_kernel<<<grid, kBlock, 0, s>>>(q);
+  if (agg) emb_bsort_scatter2_kernel<<<c->num_sms * 2, kBlock, ssm, s>>>(q);
+  else emb_bsort_scatter_kernel<<<grid, kBlock, 0, s>>>(q);
   void (*k)(SortParams) = nullptr;
   if (c->bvb == 8) k = emb_bsort_reduce_kernel<8, 1>;
   else if (c->bnv == 2) k = emb_bsort_reduce_kernel<16, 2>;
@@ -981,7 +993,7 @@ emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* i
   c->bwd_ready_pending = false;
   BwdParams p;
   fill_bwd_params(c, &p);
-  if (c->bwd_algo == 1 && c->T_r > 0 && c->T_r <= 2048)
+  if (c->bwd_algo >= 1 && c->T_r > 0 && c->T_r <= 2048)
     return backward_sorted(c, p, offsets, indices, s);
   p.offsets = offsets;
   p.indices = indices;
@@ -1135,7 +1147,7 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "bwd_v2")) c->bwd_v2 = v ? 1 : 0;
-  else if (!strcmp(key, "bwd_algo")) { if (v != 0 && v != 1) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0 or 1"); c->bwd_algo = (int)v; }
+  else if (!strcmp(key, "bwd_algo")) { if (v < 0 || v > 2) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0, 1 or 2"); c->bwd_algo = (int)v; }
   else if (!strcmp(key, "bwd_max_nnz")) {
     if (v < 0 || v >= (1ll << 32)) FAIL(c, EMB_ERR_ARG, "bwd_max_nnz not in [0, 2^32)");
     if (c->d_pairs) { cudaFree(c->d_pairs); c->d_pairs = nullptr; }

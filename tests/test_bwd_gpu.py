@@ -107,7 +107,8 @@ def test_bwd_placement_invariance():
                                   {"bwd_group": 7}, {"bwd_group": 1}, {"bwd_v2": 1}, {"bwd_v2": 1, "bwd_group": 3},
                                   {"bwd_v2": 1, "bwd_interleave": 0}, {"bwd_v2": 1, "bwd_cache": 8},
                                   {"bwd_v2": 1, "bwd_cache": 16, "bwd_chunk_rows": 1024},
-                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}, {"bwd_algo": 1}])
+                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}, {"bwd_algo": 1},
+                                  {"bwd_algo": 2}])
 def test_bwd_chunk_orders_integer_exact(opts):
     """every chunk order (table-major, groups of g tables incl. a ragged last group, all
     tables interleaved) visits every bag exactly once: exact on integer gradients"""
@@ -139,13 +140,14 @@ def test_bwd_row_cache_exact_and_float_bound(dim, cache):
         assert np.all(err <= n * 2.0 ** -24 * 2 * S[t] + 1e-30), t
 
 
-@pytest.mark.parametrize("G,dist", [(1, "zipf"), (2, "uniform"), (3, "zipf")])
-def test_bwd_sorted_algo_integer_exact_multi_epoch(G, dist):
+@pytest.mark.parametrize("G,dist,algo", [(1, "zipf", 1), (2, "uniform", 1), (3, "zipf", 1), (1, "zipf", 2),
+                                          (2, "uniform", 2), (3, "zipf", 2)])
+def test_bwd_sorted_algo_integer_exact_multi_epoch(G, dist, algo):
     """bwd_algo 1 (counting sort + segmented sum): exact on integer gradients over 3 epochs
     (workspace reuse, counters re-zeroed), incl. empty bags and G > 1 one-sided dY loads"""
     w = synth.make_workload("tiny", G=G, pmin=0, pmax=70, B=131, T=5, dim=128, rows=400, dist=dist)
     dY = _dY(w, 31, integer=True)
-    got, offs, idxs = _run_bwd(w, dY, 32, epochs=3, opts={"bwd_algo": 1})
+    got, offs, idxs = _run_bwd(w, dY, 32, epochs=3, opts={"bwd_algo": algo})
     ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
     for t in range(w.T):
         assert np.array_equal(got[t].astype(np.float64), 3 * ref[t]), t
