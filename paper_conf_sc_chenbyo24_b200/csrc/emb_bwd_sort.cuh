@@ -44,6 +44,12 @@ struct SortParams {
   int64_t R, cap, B, timeout_ns;
   int32_t T, T_r, d, G, rank, lanes, chunk_rows;
   uint32_t epoch;
+  // bwd_algo 3 (LSD radix sort): ping-pong entry buffers, per-(digit, tile) histogram
+  const uint2* rin;
+  uint2* rout;
+  uint32_t* ghist;             // [256][nblk_r], digit-major
+  int64_t nblk_r;
+  int32_t shift;
 };
 
 constexpr int kScanTile = 4096;    // counters per scan tile (256 threads x 16)
@@ -427,6 +433,110 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_scatter2_kernel(const __grid
       hk[i] = kHashEmpty;
       hc[i] = 0;
     }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------------------- bwd_algo 3
+// LSD radix sort of the {code, g} entries by g, 8-bit digits: per pass an upsweep writes
+// each tile's 256-bin digit histogram (shared-memory atomics only), an exclusive scan over
+// the digit-major [256][tiles] matrix gives every (digit, tile) its output offset, and a
+// stable downsweep ranks each tile's entries per digit (match.any within a warp, per-warp
+// digit counts in shared memory across warps and iterations) and scatters them.  No
+// global atomics on row counters at all.
+constexpr int kRTile = 4096;       // entries per tile (256 threads x 16, striped)
+
+// entries in position order: pairs[j] = {dY row code of j's bag, global row of j}
+__global__ void __launch_bounds__(kBlock) emb_bradix_gen_kernel(const __grid_constant__ SortParams p) {
+  __shared__ int64_t ofs[kBlock / 32][33];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t B = p.B, nbags = (int64_t)p.T_r * B;
+  if (nbags == 0) return;
+  const int64_t nnz = sort_nnz(p);
+  if (nnz > p.cap) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr(&p.ctrl->err, 0x4u);
+    return;
+  }
+  const int64_t cb64 = nnz > 0 ? ((int64_t)p.chunk_rows * nbags + nnz - 1) / nnz : 31;
+  const int cb = (int)(cb64 < 1 ? 1 : (cb64 > 31 ? 31 : cb64));
+  const int64_t cpt = (B + cb - 1) / cb, nchunks = cpt * p.T_r;
+  const int64_t nw = (int64_t)gridDim.x * (kBlock / 32);
+  for (int64_t c = (int64_t)blockIdx.x * (kBlock / 32) + w; c < nchunks; c += nw) {
+    const int t_l = (int)(c / cpt);
+    const int64_t b0 = (c % cpt) * cb;
+    const int nb = (int)min((int64_t)cb, B - b0);
+    if (lane <= nb) ofs[w][lane] = ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane);
+    __syncwarp();
+    const int64_t pos0 = ofs[w][0], pos1 = ofs[w][nb];
+    const int64_t rb = __ldg(p.rowbase + t_l);
+    const int64_t tglob = __ldg(&p.tables[t_l].tglob);
+    for (int64_t j = pos0 + lane; j < pos1; j += 32) {
+      int lo = 0, hi = nb - 1;                          // last bag with start <= j
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (ofs[w][mid] <= j) lo = mid;
+        else hi = mid - 1;
+      }
+      const int64_t b = b0 + lo;
+      int dst = 0;
+      while (b >= p.bstart[dst + 1]) ++dst;
+      const uint32_t code = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
+      p.pairs[j] = make_uint2(code, (uint32_t)(rb + ld_stream_i64(p.indices + j)));
+    }
+    __syncwarp();
+  }
+}
+
+__global__ void __launch_bounds__(kBlock) emb_bradix_up_kernel(const __grid_constant__ SortParams p) {
+  __shared__ uint32_t hist[256];
+  hist[threadIdx.x] = 0;
+  __syncthreads();
+  const int64_t nnz = sort_nnz(p);
+  const int64_t base = (int64_t)blockIdx.x * kRTile;
+  if (nnz <= p.cap) {
+#pragma unroll 4
+    for (int i = 0; i < kRTile / kBlock; ++i) {
+      const int64_t idx = base + (int64_t)i * kBlock + threadIdx.x;
+      if (idx < nnz) atomicAdd(hist + ((p.rin[idx].y >> p.shift) & 255u), 1u);
+    }
+  }
+  __syncthreads();
+  p.ghist[(int64_t)threadIdx.x * p.nblk_r + blockIdx.x] = hist[threadIdx.x];
+}
+
+__global__ void __launch_bounds__(kBlock) emb_bradix_down_kernel(const __grid_constant__ SortParams p) {
+  __shared__ uint32_t run[256];
+  __shared__ uint32_t wcnt[kBlock / 32][256];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  run[threadIdx.x] = p.ghist[(int64_t)threadIdx.x * p.nblk_r + blockIdx.x];   // scanned offsets
+#pragma unroll
+  for (int k = 0; k < kBlock / 32; ++k) wcnt[k][threadIdx.x] = 0;
+  __syncthreads();
+  const int64_t nnz = sort_nnz(p);
+  if (nnz > p.cap) return;
+  const int64_t base = (int64_t)blockIdx.x * kRTile;
+  const unsigned lt = (1u << lane) - 1u;
+  for (int i = 0; i < kRTile / kBlock; ++i) {
+    const int64_t idx = base + (int64_t)i * kBlock + threadIdx.x;
+    const bool valid = idx < nnz;
+    const uint2 e = valid ? p.rin[idx] : make_uint2(0u, 0u);
+    const uint32_t d = (e.y >> p.shift) & 255u;
+    const unsigned peers = __match_any_sync(kFull, valid ? d : (0x1000u | (uint32_t)lane));
+    if (valid && (__ffs(peers) - 1) == lane) wcnt[w][d] = (uint32_t)__popc(peers);
+    __syncthreads();
+    if (valid) {
+      uint32_t pre = run[d];
+      for (int k = 0; k < w; ++k) pre += wcnt[k][d];
+      p.rout[pre + (uint32_t)__popc(peers & lt)] = e;
+    }
+    __syncthreads();
+    uint32_t tot = 0;                                   // thread t owns digit t
+#pragma unroll
+    for (int k = 0; k < kBlock / 32; ++k) {
+      tot += wcnt[k][threadIdx.x];
+      wcnt[k][threadIdx.x] = 0;
+    }
+    run[threadIdx.x] += tot;
     __syncthreads();
   }
 }

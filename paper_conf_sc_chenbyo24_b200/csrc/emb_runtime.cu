@@ -132,6 +132,10 @@ struct emb_ctx {
   uint32_t* d_bcnt = nullptr;
   uint32_t* d_bsum = nullptr;
   uint2* d_pairs = nullptr;
+  uint2* d_pairs_b = nullptr;      // bwd_algo 3: radix-sort ping-pong buffer
+  uint32_t* d_ghist = nullptr;     // bwd_algo 3: [256][tiles] digit histograms
+  uint32_t* d_rbsum = nullptr;
+  int64_t rs_nblk = 0;
   int fwd_interleave = 0;
   int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
   int tail_div = 4;                // guided tail of the forward's chunk schedule
@@ -512,6 +516,9 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bsort_scan_apply_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scatter_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_hist2_kernel);
+    cudaFuncGetAttributes(&a, emb_bradix_gen_kernel);
+    cudaFuncGetAttributes(&a, emb_bradix_up_kernel);
+    cudaFuncGetAttributes(&a, emb_bradix_down_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scatter2_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1>);
@@ -941,6 +948,40 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   q.epoch = bp.epoch;
   const size_t tsm = (size_t)(c->T_r + 1) * 2 * sizeof(int64_t);
   const int grid = c->num_sms * 8;
+  if (c->bwd_algo == 3) {                               // LSD radix sort of the entries by row
+    if (!c->d_pairs_b) {
+      c->rs_nblk = (c->bs_cap + kRTile - 1) / kRTile;
+      const int64_t nh = 256 * c->rs_nblk;
+      CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_cap * sizeof(uint2)));
+      CK(c, cudaMalloc(&c->d_ghist, (size_t)nh * sizeof(uint32_t)));
+      CK(c, cudaMalloc(&c->d_rbsum, (size_t)((nh + kScanTile - 1) / kScanTile) * sizeof(uint32_t)));
+    }
+    emb_bradix_gen_kernel<<<grid, kBlock, 0, s>>>(q);
+    int bits = 1;
+    while (bits < 32 && (1ll << bits) < c->bs_R) ++bits;
+    const int passes = (bits + 7) / 8;
+    const int64_t nh = 256 * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
+    uint2* in = c->d_pairs;
+    uint2* out = c->d_pairs_b;
+    q.ghist = c->d_ghist;
+    q.nblk_r = c->rs_nblk;
+    SortParams qs = q;                                  // the scan runs over the histograms
+    qs.cnt = c->d_ghist;
+    qs.R = nh;
+    qs.bsum = c->d_rbsum;
+    for (int ps = 0; ps < passes; ++ps) {
+      q.rin = in;
+      q.rout = out;
+      q.shift = 8 * ps;
+      emb_bradix_up_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
+      emb_bsort_scan_sum_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
+      emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_rbsum, nb2);
+      emb_bsort_scan_apply_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
+      emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
+      std::swap(in, out);
+    }
+    q.pairs = in;                                       // sorted by row
+  } else {
   CK(c, cudaMemsetAsync(c->d_bcnt, 0, (size_t)c->bs_R * sizeof(uint32_t), s));
   const bool agg = c->bwd_algo == 2;                   // CTA-level shared-memory aggregation
   const size_t hsm = (size_t)2 * kHashSlots * sizeof(uint32_t) + tsm;
@@ -959,6 +1000,7 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   }
   if (agg) emb_bsort_scatter2_kernel<<<c->num_sms * 2, kBlock, ssm, s>>>(q);
   else emb_bsort_scatter_kernel<<<grid, kBlock, 0, s>>>(q);
+  }
   void (*k)(SortParams) = nullptr;
   if (c->bvb == 8) k = emb_bsort_reduce_kernel<8, 1>;
   else if (c->bnv == 2) k = emb_bsort_reduce_kernel<16, 2>;
@@ -1073,6 +1115,9 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->d_bcnt) cudaFree(c->d_bcnt);
   if (c->d_bsum) cudaFree(c->d_bsum);
   if (c->d_pairs) cudaFree(c->d_pairs);
+  if (c->d_pairs_b) cudaFree(c->d_pairs_b);
+  if (c->d_ghist) cudaFree(c->d_ghist);
+  if (c->d_rbsum) cudaFree(c->d_rbsum);
   if (c->s_out) cudaStreamDestroy(c->s_out);
   delete c;
   return st;
@@ -1147,10 +1192,13 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "bwd_v2")) c->bwd_v2 = v ? 1 : 0;
-  else if (!strcmp(key, "bwd_algo")) { if (v < 0 || v > 2) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0, 1 or 2"); c->bwd_algo = (int)v; }
+  else if (!strcmp(key, "bwd_algo")) { if (v < 0 || v > 3) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0, 1, 2 or 3"); c->bwd_algo = (int)v; }
   else if (!strcmp(key, "bwd_max_nnz")) {
     if (v < 0 || v >= (1ll << 32)) FAIL(c, EMB_ERR_ARG, "bwd_max_nnz not in [0, 2^32)");
     if (c->d_pairs) { cudaFree(c->d_pairs); c->d_pairs = nullptr; }
+    if (c->d_pairs_b) { cudaFree(c->d_pairs_b); c->d_pairs_b = nullptr; }
+    if (c->d_ghist) { cudaFree(c->d_ghist); c->d_ghist = nullptr; }
+    if (c->d_rbsum) { cudaFree(c->d_rbsum); c->d_rbsum = nullptr; }
     c->bs_cap = v;
   }
   else if (!strcmp(key, "bwd_cache")) {

@@ -108,7 +108,7 @@ def test_bwd_placement_invariance():
                                   {"bwd_v2": 1, "bwd_interleave": 0}, {"bwd_v2": 1, "bwd_cache": 8},
                                   {"bwd_v2": 1, "bwd_cache": 16, "bwd_chunk_rows": 1024},
                                   {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}, {"bwd_algo": 1},
-                                  {"bwd_algo": 2}])
+                                  {"bwd_algo": 2}, {"bwd_algo": 3}])
 def test_bwd_chunk_orders_integer_exact(opts):
     """every chunk order (table-major, groups of g tables incl. a ragged last group, all
     tables interleaved) visits every bag exactly once: exact on integer gradients"""
@@ -121,11 +121,11 @@ def test_bwd_chunk_orders_integer_exact(opts):
 
 
 @pytest.mark.parametrize("dim,cache", [(16, 8), (64, 16), (128, 32), (256, 8), (16, -1), (64, -1), (128, -1),
-                                       (256, -1), (512, -1)])
+                                       (256, -1), (512, -1), (64, -3), (128, -3)])
 def test_bwd_row_cache_exact_and_float_bound(dim, cache):
     """f2 per-warp dW row cache (bwd_cache): integer gradients exact, float gradients within
     the order-independent summation bound (cached rows are summed in shared memory first)"""
-    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512} if cache > 0 else {"bwd_algo": 1}
+    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512} if cache > 0 else {"bwd_algo": -cache}
     w = synth.make_workload("tiny", G=2, pmin=0, pmax=60, B=150, T=3, dim=dim, rows=200, dist="zipf")
     got, offs, idxs = _run_bwd(w, _dY(w, 21, integer=True), 22, opts=opts)
     ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, _dY(w, 21, integer=True), w.B, w.G)
@@ -141,7 +141,8 @@ def test_bwd_row_cache_exact_and_float_bound(dim, cache):
 
 
 @pytest.mark.parametrize("G,dist,algo", [(1, "zipf", 1), (2, "uniform", 1), (3, "zipf", 1), (1, "zipf", 2),
-                                          (2, "uniform", 2), (3, "zipf", 2)])
+                                          (2, "uniform", 2), (3, "zipf", 2), (1, "zipf", 3), (2, "uniform", 3),
+                                          (3, "zipf", 3)])
 def test_bwd_sorted_algo_integer_exact_multi_epoch(G, dist, algo):
     """bwd_algo 1 (counting sort + segmented sum): exact on integer gradients over 3 epochs
     (workspace reuse, counters re-zeroed), incl. empty bags and G > 1 one-sided dY loads"""
