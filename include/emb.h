@@ -210,7 +210,7 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * sync) or preset by "bwd_max_nnz"; a later CSR with more lookups sets
  * EMB_DEVERR_CAPACITY and skips the step; 2 = the same with the histogram and the scatter
  * aggregated per CTA in a shared-memory hash table first; 3 = the entries sorted by row with
- * an LSD radix sort (8-bit digits, per-tile shared-memory histograms, stable scatter) instead
+ * an LSD radix sort (9-bit digits, per-tile shared-memory histograms, stable staged scatter) instead
  * of per-row counters: 2 more entry buffers of 8 B per lookup),
  * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
  * of that many records and makes every warp append {globaltimer ns, bytes stored to

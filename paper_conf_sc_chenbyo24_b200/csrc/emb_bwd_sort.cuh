@@ -438,13 +438,13 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_scatter2_kernel(const __grid
 }
 
 // ---------------------------------------------------------------------------- bwd_algo 3
-// LSD radix sort of the {code, g} entries by g, 8-bit digits: per pass an upsweep writes
-// each tile's 256-bin digit histogram (shared-memory atomics only), an exclusive scan over
-// the digit-major [256][tiles] matrix gives every (digit, tile) its output offset, and a
+// LSD radix sort of the {code, g} entries by g, 9-bit digits: per pass an upsweep writes
+// each tile's 512-bin digit histogram (shared-memory atomics only), an exclusive scan over
+// the digit-major [512][tiles] matrix gives every (digit, tile) its output offset, and a
 // stable downsweep ranks each tile's entries per digit (match.any within a warp, per-warp
 // digit counts in shared memory across warps and iterations) and scatters them.  No
 // global atomics on row counters at all.
-constexpr int kRTile = 4096;       // entries per tile (256 threads x 16, striped)
+constexpr int kRTile = 4096;       // entries per tile (8 warps x 512 contiguous)
 
 // entries in position order: pairs[j] = {dY row code of j's bag, global row of j}
 __global__ void __launch_bounds__(kBlock) emb_bradix_gen_kernel(const __grid_constant__ SortParams p) {
@@ -487,9 +487,12 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_gen_kernel(const __grid_con
   }
 }
 
+constexpr int kRBits = 9;                      // digit width: 3 passes cover 27-bit rows
+constexpr int kRBins = 1 << kRBits;
+
 __global__ void __launch_bounds__(kBlock) emb_bradix_up_kernel(const __grid_constant__ SortParams p) {
-  __shared__ uint32_t hist[256];
-  hist[threadIdx.x] = 0;
+  __shared__ uint32_t hist[kRBins];
+  for (int d = threadIdx.x; d < kRBins; d += kBlock) hist[d] = 0;
   __syncthreads();
   const int64_t nnz = sort_nnz(p);
   const int64_t base = (int64_t)blockIdx.x * kRTile;
@@ -497,47 +500,95 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_up_kernel(const __grid_cons
 #pragma unroll 4
     for (int i = 0; i < kRTile / kBlock; ++i) {
       const int64_t idx = base + (int64_t)i * kBlock + threadIdx.x;
-      if (idx < nnz) atomicAdd(hist + ((p.rin[idx].y >> p.shift) & 255u), 1u);
+      if (idx < nnz) atomicAdd(hist + ((p.rin[idx].y >> p.shift) & (kRBins - 1)), 1u);
     }
   }
   __syncthreads();
-  p.ghist[(int64_t)threadIdx.x * p.nblk_r + blockIdx.x] = hist[threadIdx.x];
+  for (int d = threadIdx.x; d < kRBins; d += kBlock) p.ghist[(int64_t)d * p.nblk_r + blockIdx.x] = hist[d];
 }
 
+// stable downsweep: each warp ranks its own contiguous 512 entries with warp-private digit
+// counters (match.any groups, the leader's shared-memory atomicAdd returns the group's
+// base: no block barrier per step), one block pass turns the counters into per-(warp,
+// digit) offsets inside the tile, the tile is staged in shared memory in digit order and
+// each digit's run is written out as consecutive 8-B entries (coalesced)
 __global__ void __launch_bounds__(kBlock) emb_bradix_down_kernel(const __grid_constant__ SortParams p) {
-  __shared__ uint32_t run[256];
-  __shared__ uint32_t wcnt[kBlock / 32][256];
+  extern __shared__ __align__(16) uint32_t rd_smem[];
+  uint2* stage = reinterpret_cast<uint2*>(rd_smem);                 // [kRTile]
+  uint32_t* lstart = rd_smem + 2 * kRTile;                          // [kRBins] tile-local digit start
+  uint32_t* gofs = lstart + kRBins;                                 // [kRBins] global start (scanned)
+  uint32_t* wcnt = gofs + kRBins;                                   // [kBlock/32][kRBins]
+  __shared__ uint32_t sh[kBlock / 32];
+  constexpr int KI = kRTile / kBlock;                               // 16 entries per lane
+  constexpr int NW = kBlock / 32;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  run[threadIdx.x] = p.ghist[(int64_t)threadIdx.x * p.nblk_r + blockIdx.x];   // scanned offsets
+  for (int d = threadIdx.x; d < kRBins; d += kBlock) {
+    gofs[d] = p.ghist[(int64_t)d * p.nblk_r + blockIdx.x];
 #pragma unroll
-  for (int k = 0; k < kBlock / 32; ++k) wcnt[k][threadIdx.x] = 0;
+    for (int k = 0; k < NW; ++k) wcnt[k * kRBins + d] = 0;
+  }
   __syncthreads();
   const int64_t nnz = sort_nnz(p);
   if (nnz > p.cap) return;
-  const int64_t base = (int64_t)blockIdx.x * kRTile;
+  const int64_t wbase = (int64_t)blockIdx.x * kRTile + (int64_t)w * (32 * KI);   // warp-contiguous
   const unsigned lt = (1u << lane) - 1u;
-  for (int i = 0; i < kRTile / kBlock; ++i) {
-    const int64_t idx = base + (int64_t)i * kBlock + threadIdx.x;
-    const bool valid = idx < nnz;
-    const uint2 e = valid ? p.rin[idx] : make_uint2(0u, 0u);
-    const uint32_t d = (e.y >> p.shift) & 255u;
-    const unsigned peers = __match_any_sync(kFull, valid ? d : (0x1000u | (uint32_t)lane));
-    if (valid && (__ffs(peers) - 1) == lane) wcnt[w][d] = (uint32_t)__popc(peers);
-    __syncthreads();
-    if (valid) {
-      uint32_t pre = run[d];
-      for (int k = 0; k < w; ++k) pre += wcnt[k][d];
-      p.rout[pre + (uint32_t)__popc(peers & lt)] = e;
-    }
-    __syncthreads();
-    uint32_t tot = 0;                                   // thread t owns digit t
+  uint2 e[KI];
+  uint32_t rk[KI];
 #pragma unroll
-    for (int k = 0; k < kBlock / 32; ++k) {
-      tot += wcnt[k][threadIdx.x];
-      wcnt[k][threadIdx.x] = 0;
+  for (int i = 0; i < KI; ++i) {
+    const int64_t idx = wbase + 32 * i + lane;
+    e[i] = idx < nnz ? p.rin[idx] : make_uint2(0u, 0xffffffffu);
+  }
+#pragma unroll
+  for (int i = 0; i < KI; ++i) {
+    const bool valid = wbase + 32 * i + lane < nnz;
+    const uint32_t d = (e[i].y >> p.shift) & (kRBins - 1);
+    const unsigned peers = __match_any_sync(kFull, valid ? d : (0x10000u | (uint32_t)lane));
+    const int leader = __ffs(peers) - 1;
+    uint32_t b = 0;
+    if (valid && leader == lane) b = atomicAdd(wcnt + w * kRBins + d, (uint32_t)__popc(peers));
+    rk[i] = __shfl_sync(kFull, b, leader) + (uint32_t)__popc(peers & lt);
+  }
+  __syncthreads();
+  {                                                      // per-(warp, digit) offsets, digit starts
+    constexpr int DP = kRBins / kBlock;
+    uint32_t tot[DP], sum = 0;
+#pragma unroll
+    for (int k = 0; k < DP; ++k) {
+      const int d = threadIdx.x * DP + k;
+      uint32_t run = 0;
+#pragma unroll
+      for (int q = 0; q < NW; ++q) {
+        const uint32_t c = wcnt[q * kRBins + d];
+        wcnt[q * kRBins + d] = run;
+        run += c;
+      }
+      tot[k] = run;
+      sum += run;
     }
-    run[threadIdx.x] += tot;
-    __syncthreads();
+    uint32_t all;
+    uint32_t ex = block_exscan(sum, sh, &all);
+#pragma unroll
+    for (int k = 0; k < DP; ++k) {
+      lstart[threadIdx.x * DP + k] = ex;
+      ex += tot[k];
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < KI; ++i) {
+    if (wbase + 32 * i + lane < nnz) {
+      const uint32_t d = (e[i].y >> p.shift) & (kRBins - 1);
+      stage[lstart[d] + wcnt[w * kRBins + d] + rk[i]] = e[i];
+    }
+  }
+  __syncthreads();
+  const int64_t base = (int64_t)blockIdx.x * kRTile;
+  const int cnt = (int)min((int64_t)kRTile, nnz - base);
+  for (int k = threadIdx.x; k < cnt; k += kBlock) {      // digit runs leave contiguously
+    const uint2 v = stage[k];
+    const uint32_t d = (v.y >> p.shift) & (kRBins - 1);
+    p.rout[gofs[d] + (uint32_t)k - lstart[d]] = v;
   }
 }
 

@@ -951,7 +951,7 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   if (c->bwd_algo == 3) {                               // LSD radix sort of the entries by row
     if (!c->d_pairs_b) {
       c->rs_nblk = (c->bs_cap + kRTile - 1) / kRTile;
-      const int64_t nh = 256 * c->rs_nblk;
+      const int64_t nh = (int64_t)kRBins * c->rs_nblk;
       CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_cap * sizeof(uint2)));
       CK(c, cudaMalloc(&c->d_ghist, (size_t)nh * sizeof(uint32_t)));
       CK(c, cudaMalloc(&c->d_rbsum, (size_t)((nh + kScanTile - 1) / kScanTile) * sizeof(uint32_t)));
@@ -959,8 +959,10 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
     emb_bradix_gen_kernel<<<grid, kBlock, 0, s>>>(q);
     int bits = 1;
     while (bits < 32 && (1ll << bits) < c->bs_R) ++bits;
-    const int passes = (bits + 7) / 8;
-    const int64_t nh = 256 * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
+    const int passes = (bits + kRBits - 1) / kRBits;
+    const int64_t nh = (int64_t)kRBins * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
+    const size_t dsm = (size_t)(2 * kRTile + (2 + kBlock / 32) * kRBins) * sizeof(uint32_t);
+    CK(c, cudaFuncSetAttribute(emb_bradix_down_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm));
     uint2* in = c->d_pairs;
     uint2* out = c->d_pairs_b;
     q.ghist = c->d_ghist;
@@ -972,12 +974,12 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
     for (int ps = 0; ps < passes; ++ps) {
       q.rin = in;
       q.rout = out;
-      q.shift = 8 * ps;
+      q.shift = kRBits * ps;
       emb_bradix_up_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
       emb_bsort_scan_sum_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
       emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_rbsum, nb2);
       emb_bsort_scan_apply_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
-      emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
+      emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, dsm, s>>>(q);
       std::swap(in, out);
     }
     q.pairs = in;                                       // sorted by row

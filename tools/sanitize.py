@@ -52,16 +52,17 @@ for G in (1, 2):
     for r in range(G):
         layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
     torch.cuda.synchronize()
-    # second backward algorithm (counting sort + segmented sum), same slots and flags
-    for r in range(G):
-        E.emb_set_option(layers[r].ctx, "bwd_algo", 1)
-        with torch.cuda.stream(streams[r]):
-            layers[r].grad_slot(streams[r]).fill_(1.0)
-        layers[r].grad_ready(streams[r])
-    torch.cuda.synchronize()
-    for r in range(G):
-        layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
-    torch.cuda.synchronize()
+    # sorted backward algorithms (counting sort / radix sort + segmented sum), same slots and flags
+    for algo in (1, 3):
+        for r in range(G):
+            E.emb_set_option(layers[r].ctx, "bwd_algo", algo)
+            with torch.cuda.stream(streams[r]):
+                layers[r].grad_slot(streams[r]).fill_(1.0)
+            layers[r].grad_ready(streams[r])
+        torch.cuda.synchronize()
+        for r in range(G):
+            layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
+        torch.cuda.synchronize()
     if G == 1:
         ho, hx = torch.from_numpy(offs[0]).pin_memory(), torch.from_numpy(idxs[0]).pin_memory()
         hout = torch.empty((w.B, w.T, w.dim)).pin_memory()
