@@ -187,7 +187,8 @@ emb_status_t emb_local_batch(const emb_ctx_t* ctx, int rank, int64_t* start, int
 emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
 
 /* Tunables (take effect on the next launch): "chunk_rows" (target rows per claimed
- * work chunk, default 256), "ctas_per_sm" (0 = occupancy max), "stagger" (1 =
+ * work chunk; 0 = auto, the default: 192 for fp32 rows and 256 for bf16 rows in the
+ * forward, 256 in the backward), "ctas_per_sm" (0 = occupancy max), "stagger" (1 =
  * destination-staggered chunk order, default), "timeout_ms" (peer wait, default
  * 10000 or env EMB_TIMEOUT_MS), "unroll" (row pipeline: 0 = auto (default), 2 or 4 = rows per group of the
  * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
