@@ -201,7 +201,7 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * "enable_backward" (f2: 1 before emb_register_tables adds two fp32 grad slots
  * [B_r][T][d] to the symmetric buffer for emb_backward), f2 backward tunables:
  * "bwd_interleave" (1 = chunks interleaved across tables, default; 0 = table-major),
- * "bwd_group" (tables interleaved at a time, default 4; 0 = all local tables),
+ * "bwd_group" (tables interleaved at a time, default 8; 0 = all local tables),
  * "bwd_v2" (1 = distinct rows of a slice scattered from a compacted shared-memory list,
  * default), "bwd_cache" (per-warp shared-memory dW row cache slots: 0, 8, 16 (default)
  * or 32; needs bwd_v2 and one vector per lane), "bwd_chunk_rows" (0 = chunk_rows),

@@ -125,7 +125,7 @@ struct emb_ctx {
   int bwd_v2 = 1;                  // backward slice scatter from a compacted smem list
   int bwd_cache = 16;              // per-warp dW row cache slots (0 off; 8 / 16 / 32; needs bwd_v2)
   int bwd_chunk_rows = 0;          // backward chunk target rows (0: chunk_rows)
-  int bwd_group = 4;               // tables interleaved at a time in the backward (0: all T_r)
+  int bwd_group = 8;               // tables interleaved at a time in the backward (0: all T_r)
   int bwd_algo = 0;                // 0: atomic scatter per bag slice; 1: counting sort + segmented sum
   int64_t bs_cap = 0, bs_R = 0, bs_nblk = 0;   // bwd_algo 1 workspace
   int64_t* d_rowbase = nullptr;
