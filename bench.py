@@ -313,6 +313,15 @@ def run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq
             "lookup_counted": {"bytes": lookup_bytes, "achieved": lookup_bytes / (ms * 1e-3) / 1e9,
                                "frac": lookup_bytes / (ms * 1e-3) / 1e9 / peak},
             "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs", "t_roof_ms": max(t_hbm, t_nvl) * 1e3}
+    if not args.opt:                                       # default kernel only: ncu of that kernel
+        try:
+            with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+                tb = json.load(f).get(f"{w.name}:{w.dist}:G{N}:backward")
+            if tb:
+                roof["traffic"] = tb["dram_bytes_per_launch"]
+                roof["traffic_source"] = tb.get("source")
+        except (OSError, ValueError):
+            pass
     layer.close()
     if N > 1:
         dist.barrier()
