@@ -61,13 +61,18 @@ typedef enum {
 typedef enum { EMB_F32 = 0, EMB_BF16 = 1 } emb_dtype_t;
 
 /* emb_forward / emb_baseline_pool flags */
-#define EMB_FWD_CHECK_BOUNDS 0x1u  /* skip indices outside [0, rows) and set EMB_DEVERR_BOUNDS */
+#define EMB_FWD_CHECK_BOUNDS 0x1u  /* skip indices outside [0, M_t) and set EMB_DEVERR_BOUNDS */
 #define EMB_FWD_SEPARATE_WAIT 0x2u /* fused kernel only signals; call emb_wait() to complete  */
 
 /* sticky device error word bits (emb_query_device_error) */
 #define EMB_DEVERR_TIMEOUT 0x1u
 #define EMB_DEVERR_BOUNDS 0x2u
 #define EMB_DEVERR_CAPACITY 0x4u /* emb_backward (bwd_algo 1): more lookups than the entry workspace; step skipped */
+
+/* Index width (SURVEY reading C12).  The paper's listing passes int64 offsets and indices
+ * (Listing 2), the default of every call below.  The *_i32 entry points take the
+ * same CSR as int32 arrays (offsets[T_r*B] < 2^31): half the index bytes in HBM and over
+ * PCIe, identical results. */
 
 /* All-gather over the caller's process group.  send: `bytes` bytes of this rank;
  * recv: world_size*bytes, rank order.  Return 0 on success.  Called only from
@@ -87,6 +92,10 @@ typedef struct {
   int32_t grid, block;        /* fused kernel launch shape                    */
   int32_t lanes, vec_bytes, vecs_per_lane; /* row-gather tiling                */
   int64_t out_slot_bytes;     /* B_r*T*d*e_o                                  */
+  int32_t out_slots;          /* depth of the symmetric output ring (3)       */
+  int32_t fwd_launches;       /* kernels one emb_forward launches             */
+  int32_t bwd_launches;       /* kernels one emb_backward launches            */
+  int32_t reserved;
 } emb_info_t;
 
 /* Create a context for `rank` of `world_size` on CUDA device `cuda_device`.
@@ -110,7 +119,7 @@ emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_f
  *   local_weights[T_r] : device pointers of this rank's tables in ascending global id,
  *                row-major [M_t][d], 16-byte aligned; zero-copy: the caller keeps them
  *                alive until emb_finalize.
- * Allocates the symmetric output (2 slots of [B_r][T][d]) + flag words, exchanges IPC
+ * Allocates the symmetric output (a ring of 3 slots of [B_r][T][d]) + flag words, exchanges IPC
  * handles through `allgather`, maps every peer.  Errors: EMB_ERR_ARG, EMB_ERR_STATE
  * (already registered), EMB_ERR_CUDA/NOMEM, EMB_ERR_PEER. */
 emb_status_t emb_register_tables(emb_ctx_t* ctx, int32_t num_tables, const int64_t* rows, const int32_t* owner,
@@ -128,9 +137,9 @@ emb_status_t emb_register_tables(emb_ctx_t* ctx, int32_t num_tables, const int64
  * in the same order, the FULL bag list of its table with GLOBAL row ids; the kernel skips
  * other shards' ids (in-kernel partitioning), stores each bag's fp32 partial sum into the
  * owner's partial slot (one-sided, like the pooled vectors), and after the exchange a
- * combine kernel sums the partials in shard order into Y_r (bf16 out: RNE once).  Not
- * supported with row-sharded tables: EMB_FWD_CHECK_BOUNDS, the comparison path,
- * backward.  Errors as emb_register_tables. */
+ * combine kernel sums the partials in shard order into Y_r (bf16 out: RNE once).
+ * EMB_FWD_CHECK_BOUNDS checks ids against the whole table's [0, rows[t]).  Not supported
+ * with row-sharded tables: the comparison path, backward.  Errors as emb_register_tables. */
 emb_status_t emb_register_sharded_tables(emb_ctx_t* ctx, int32_t num_tables, const int64_t* rows,
                                          const int32_t* num_shards, const int32_t* shard_owner,
                                          const int64_t* shard_row_start, int32_t dim, emb_dtype_t weight_dtype,
@@ -142,16 +151,24 @@ emb_status_t emb_register_sharded_tables(emb_ctx_t* ctx, int32_t num_tables, con
  *             indices[offsets[t_l*B+b] .. offsets[t_l*B+b+1]) (C11; L212-215)
  *   indices : device int64 local row ids in [0, M_t) (C1, C12)
  *   *out    : receives the device pointer of Y_r = [B_r][T][d] (out dtype) for this
- *             epoch; library-owned, valid until the 2nd subsequent emb_forward or
- *             emb_finalize.  The output of epoch e must be consumed on `stream`
- *             (or a stream ordered after it) before this rank's forward e+2.
+ *             epoch e; library-owned slot e % 3 of the symmetric ring.  Every read of it
+ *             must be ordered before this rank's forward e+2 is launched (on `stream`,
+ *             or on another stream that `stream` waits on before that launch): a peer
+ *             can overwrite the slot with its forward e+3 as soon as this rank's forward
+ *             e+2 has signalled.  Valid until then or emb_finalize.
  * Without EMB_FWD_SEPARATE_WAIT the kernel completes only when every peer's
  * pooled vectors for this rank have landed (in-kernel acquire wait), so any later
- * work on `stream` sees the whole Y_r.  Empty bags produce +0.0 (C2).
+ * work on `stream` sees the whole Y_r.  With it, emb_wait completes the forward; a
+ * forward issued while the previous one's emb_wait is still due enqueues that wait
+ * first.  Empty bags produce +0.0 (C2).  IEEE fp32 adds, no flush-to-zero; NaN and
+ * Inf propagate (C7).  Unknown flag bits: EMB_ERR_ARG.
  * Errors: EMB_ERR_STATE (not registered), EMB_ERR_ARG, EMB_ERR_CUDA.  Device-side
  * failures (peer timeout, bounds) set the sticky device error word instead. */
 emb_status_t emb_forward(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, uint32_t flags,
                          void* stream, void** out);
+/* emb_forward with int32 offsets / indices (C12 option, see above). */
+emb_status_t emb_forward_i32(emb_ctx_t* ctx, const int32_t* offsets, const int32_t* indices, uint32_t flags,
+                             void* stream, void** out);
 
 /* Complete a forward issued with EMB_FWD_SEPARATE_WAIT: enqueue the acquire wait on
  * every peer's flag for the latest epoch on `stream`. */
@@ -167,13 +184,18 @@ emb_status_t emb_forward_host(emb_ctx_t* ctx, const int64_t* h_offsets, const in
 
 /* Pipelined end-to-end path (same inputs/outputs as emb_forward_host): call k's H2D
  * (internal copy-in stream, two alternating device stages) overlaps call k-1's kernel
- * (on `stream`) and call k-2's D2H (internal copy-out stream).  h_out of a call is
+ * (on `stream`) and call k-1's D2H (internal copy-out stream); the forward of call k
+ * waits for the D2H of call k-2 (output-ring rule of emb_forward).  The peer wait is
+ * always in-kernel here (EMB_FWD_SEPARATE_WAIT is ignored).  h_out of a call is
  * complete once emb_host_drain(ctx, s) has been called and `s` synchronized (or after a
  * later call's drain).  The host input buffers of a call must stay unchanged, and its
  * h_out must not be reused by another in-flight call, until then; h_out buffers should
  * be pinned.  Two calls in flight at most per stage (the library waits on events). */
 emb_status_t emb_forward_host_async(emb_ctx_t* ctx, const int64_t* h_offsets, const int64_t* h_indices,
                                     uint32_t flags, void* stream, void* h_out);
+/* Same with int32 host offsets / indices (C12 option). */
+emb_status_t emb_forward_host_async_i32(emb_ctx_t* ctx, const int32_t* h_offsets, const int32_t* h_indices,
+                                        uint32_t flags, void* stream, void* h_out);
 
 /* Make `stream` wait for every outstanding copy of emb_forward_host_async. */
 emb_status_t emb_host_drain(emb_ctx_t* ctx, void* stream);
@@ -190,11 +212,10 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * work chunk; 0 = auto, the default: 192 for fp32 rows and 256 for bf16 rows in the
  * forward, 256 in the backward), "ctas_per_sm" (0 = occupancy max), "stagger" (1 =
  * destination-staggered chunk order, default), "timeout_ms" (peer wait, default
- * 10000 or env EMB_TIMEOUT_MS), "unroll" (row pipeline: 0 = auto (default), 2 or 4 = rows per group of the
- * register pipeline for 16-byte lane vectors (2 implies 6 CTAs/SM); 8 or 16 = rows in
- * flight per warp in a cp.async shared-memory ring), "minblocks" (CTAs of 256 per
- * SM the register budget is sized for: 0 = auto (5 for fp32 rows of one 16-B vector per lane,
- * 4 for other one-vector-per-lane tiles, else 1), 1, 4, 5, 6).
+ * 10000 or env EMB_TIMEOUT_MS), "fwd_interleave" (1 = forward chunks interleaved across
+ * tables instead of table-major), "tail_div" (the last table's chunks are this many times
+ * smaller, default 4; 1 = off), "carveout" (shared-memory carve-out percent; 0 = auto, the
+ * default: the smallest that fits the kernel's occupancy; -1 = driver default),
  * "tma_store" (f4, PAPER.md L386 aggregated stores: 1 = pooled vectors are staged per
  * warp in shared memory and shipped 4 at a time to 4 arbitrary output rows with one TMA
  * scatter4; needs full-warp rows with one vector per lane and d <= 256),
@@ -202,17 +223,15 @@ emb_status_t emb_get_info(const emb_ctx_t* ctx, emb_info_t* info);
  * [B_r][T][d] to the symmetric buffer for emb_backward), f2 backward tunables:
  * "bwd_interleave" (1 = chunks interleaved across tables, default; 0 = table-major),
  * "bwd_group" (tables interleaved at a time, default 8; 0 = all local tables),
- * "bwd_v2" (1 = distinct rows of a slice scattered from a compacted shared-memory list,
- * default), "bwd_cache" (per-warp shared-memory dW row cache slots: 0, 8, 16 (default)
- * or 32; needs bwd_v2 and one vector per lane), "bwd_chunk_rows" (0 = chunk_rows),
- * "bwd_algo" (0 = atomic scatter per bag slice; 1 = counting sort of the lookups by dW
- * row + segmented gather-sum, one red.add per run of equal rows: library-owned workspace
- * of 4 B per local row + 8 B per lookup, sized on the first call from the CSR (one host
- * sync) or preset by "bwd_max_nnz"; a later CSR with more lookups sets
- * EMB_DEVERR_CAPACITY and skips the step; 2 = the same with the histogram and the scatter
- * aggregated per CTA in a shared-memory hash table first; 3 = the entries sorted by row with
- * an LSD radix sort (9-bit digits, per-tile shared-memory histograms, stable staged scatter) instead
- * of per-row counters: 2 more entry buffers of 8 B per lookup),
+ * "bwd_cache" (per-warp shared-memory dW row cache: 16 slots (default) or 0; rows of one
+ * vector per lane), "bwd_chunk_rows" (0 = chunk_rows),
+ * "bwd_algo" (0 = atomic scatter per bag slice, default; 1 = LSD radix sort of the lookups
+ * by dW row + segmented gather-sum, one red.add per run of equal rows: library-owned
+ * workspace of 16 B per lookup, sized on the first call from the CSR (one host sync) or
+ * preset by "bwd_max_nnz"; a later CSR with more lookups sets EMB_DEVERR_CAPACITY and
+ * skips the step; needs fewer than 2^27 local rows),
+ * "debug_d2h_delay_us" (test hook: the pipelined host path stalls its copy-out stream this
+ * long before every D2H, to exercise the output-ring rule under a slow consumer),
  * "trace_capacity" (f1 instrumentation: > 0 allocates a device buffer
  * of that many records and makes every warp append {globaltimer ns, bytes stored to
  * peers << 32 | bytes stored locally} after each claimed chunk; 0 disables).
@@ -227,7 +246,7 @@ emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
  *       enqueues a wait until every peer finished reading the slot's previous use);
  *   emb_backward_grad_ready(ctx, stream) -> releases "my dY is written" to every peer
  *       (stream-ordered after the fill);
- *   emb_backward(ctx, offsets, indices, dW, flags, stream) -> one fused kernel acquires
+ *   emb_backward(ctx, offsets, indices, dW, flags = 0, stream) -> one fused kernel acquires
  *       every peer's "ready" flag and, per local bag, loads the
  *       bag's gradient vector from the DP rank's slot (one-sided NVLink load) and
  *       atomically adds it (red.add.f32, FTZ per the hardware atomic; a warp may first
@@ -242,7 +261,8 @@ emb_status_t emb_set_option(emb_ctx_t* ctx, const char* key, int64_t value);
  * peer (emb_backward_grad_slot waits on it before a slot is refilled).
  * Requires "enable_backward" before emb_register_tables.  Errors: EMB_ERR_STATE (also for
  * emb_backward without a preceding grad_ready), EMB_ERR_ARG, EMB_ERR_CUDA; peer timeouts
- * set EMB_DEVERR_TIMEOUT. */
+ * set EMB_DEVERR_TIMEOUT.  If emb_backward fails after a grad_ready, it still releases
+ * the peers ("done" flags) and clears the pending state, so the next step can proceed. */
 emb_status_t emb_backward_grad_slot(emb_ctx_t* ctx, void* stream, void** dY);
 emb_status_t emb_backward_grad_ready(emb_ctx_t* ctx, void* stream);
 emb_status_t emb_backward(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, void* const* dW,
@@ -268,6 +288,8 @@ emb_status_t emb_baseline_splits(const emb_ctx_t* ctx, int64_t* send_counts, int
  * caller-owned device buffer send = [G][B_dst][T_r][d] (out dtype). */
 emb_status_t emb_baseline_pool(emb_ctx_t* ctx, const int64_t* offsets, const int64_t* indices, uint32_t flags,
                                void* stream, void* send);
+emb_status_t emb_baseline_pool_i32(emb_ctx_t* ctx, const int32_t* offsets, const int32_t* indices, uint32_t flags,
+                                   void* stream, void* send);
 
 /* Unpack/rearrange after the all-to-all: recv = [G][B_r][T_src][d] (blocks in
  * source-rank order, tables of each source in ascending global id) into

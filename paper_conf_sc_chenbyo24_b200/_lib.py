@@ -7,7 +7,7 @@ import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libemb.so")
-if os.environ.get("EMB_LIB"):            # experiment builds (build.build_variant) only
+if os.environ.get("EMB_LIB"):            # experiment builds (tools/variants.py) only
     LIB_PATH = os.environ["EMB_LIB"]
 
 EMB_OK, EMB_ERR_ARG, EMB_ERR_STATE, EMB_ERR_CUDA, EMB_ERR_NOMEM, EMB_ERR_PEER, EMB_ERR_TIMEOUT, EMB_ERR_BOUNDS = range(8)
@@ -18,6 +18,7 @@ EMB_FWD_CHECK_BOUNDS = 0x1
 EMB_FWD_SEPARATE_WAIT = 0x2
 EMB_DEVERR_TIMEOUT = 0x1
 EMB_DEVERR_BOUNDS = 0x2
+EMB_DEVERR_CAPACITY = 0x4
 
 ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_size_t)
 
@@ -28,7 +29,8 @@ class EmbInfo(C.Structure):
                 ("weight_dtype", C.c_int32), ("out_dtype", C.c_int32), ("global_batch", C.c_int64),
                 ("local_batch_start", C.c_int64), ("local_batch", C.c_int64), ("epoch", C.c_uint64),
                 ("grid", C.c_int32), ("block", C.c_int32), ("lanes", C.c_int32), ("vec_bytes", C.c_int32),
-                ("vecs_per_lane", C.c_int32), ("out_slot_bytes", C.c_int64)]
+                ("vecs_per_lane", C.c_int32), ("out_slot_bytes", C.c_int64), ("out_slots", C.c_int32),
+                ("fwd_launches", C.c_int32), ("bwd_launches", C.c_int32), ("reserved", C.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -43,9 +45,11 @@ SIGNATURES = {
                                               C.POINTER(C.c_int32), C.POINTER(C.c_int64), C.c_int32, C.c_int, C.c_int,
                                               C.c_int64, C.POINTER(C.c_void_p)]),
     "emb_forward": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(C.c_void_p)]),
+    "emb_forward_i32": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(C.c_void_p)]),
     "emb_wait": (C.c_int, [C.c_void_p, C.c_void_p]),
     "emb_forward_host": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
     "emb_forward_host_async": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
+    "emb_forward_host_async_i32": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
     "emb_host_drain": (C.c_int, [C.c_void_p, C.c_void_p]),
     "emb_finalize": (C.c_int, [C.c_void_p]),
     "emb_local_batch": (C.c_int, [C.c_void_p, C.c_int, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
@@ -59,6 +63,7 @@ SIGNATURES = {
     "emb_trace_read": (C.c_int, [C.c_void_p, C.c_void_p, C.c_int64, C.POINTER(C.c_int64)]),
     "emb_baseline_splits": (C.c_int, [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]),
     "emb_baseline_pool": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
+    "emb_baseline_pool_i32": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
     "emb_baseline_unpack": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
 }
 

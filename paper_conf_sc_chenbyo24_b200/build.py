@@ -16,14 +16,21 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 # no fast-math: FTZ / reassociation would break bit-exactness with the canonical oracle (C7)
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC", "-ftz=false", "-prec-div=true",
-         "-prec-sqrt=true", "-fmad=false", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
+         "-prec-sqrt=true", "-fmad=false", "-Xptxas", "-v", "--expt-relaxed-constexpr",
+         "--compress-mode=size"]   # compressed fatbin: the .so shrinks ~8x, loads the same SASS
 
 CSRC = os.path.join(PKG, "csrc")
+# the fused forward is instantiated per (weight, output) dtype pair: one source, four objects
+_PAIRS = [("f32_f32", "float", "float"), ("f32_bf16", "float", "__nv_bfloat16"),
+          ("bf16_f32", "__nv_bfloat16", "float"), ("bf16_bf16", "__nv_bfloat16", "__nv_bfloat16")]
 LIBS = {
-    "emb": dict(srcs=[os.path.join(CSRC, f) for f in ("emb_runtime.cu", "emb_inst_f32_f32.cu", "emb_inst_f32_bf16.cu",
-                                                       "emb_inst_bf16_f32.cu", "emb_inst_bf16_bf16.cu")],
-                deps=[os.path.join(CSRC, "emb_kernels.cuh"), os.path.join(CSRC, "emb_dispatch.h"), os.path.join(CSRC, "emb_bwd.cuh"), os.path.join(CSRC, "emb_bwd_sort.cuh"),
-                      os.path.join(ROOT, "include", "emb.h")],
+    "emb": dict(srcs=[os.path.join(CSRC, "emb_runtime.cu")] +
+                     [(os.path.join(CSRC, "emb_inst.cu"), f"inst_{tag}",
+                       [f"-DEMB_INST_WT={w}", f"-DEMB_INST_OT={o}", f"-DEMB_INST_NAME=pick_fwd_{tag}"])
+                      for tag, w, o in _PAIRS],
+                deps=[os.path.join(CSRC, f) for f in ("emb_kernels.cuh", "emb_dispatch.h", "emb_bwd.cuh",
+                                                      "emb_bwd_sort.cuh", "emb_inst.cu")] +
+                     [os.path.join(ROOT, "include", "emb.h")],
                 out=os.path.join(PKG, "libemb.so")),
     "synth": dict(srcs=[os.path.join(ROOT, "synth", "csrc", "synth_gen.cu")],
                   deps=[os.path.join(ROOT, "include", "synth.h")],
@@ -31,12 +38,20 @@ LIBS = {
 }
 
 
+def _src(entry):
+    """(path, object stem, extra flags) of a source entry (a path or such a tuple)."""
+    if isinstance(entry, tuple):
+        return entry
+    return entry, os.path.basename(entry), []
+
+
 def _stale(spec) -> bool:
     out = spec["out"]
     if not os.path.exists(out):
         return True
     t = os.path.getmtime(out)
-    return any(os.path.getmtime(s) > t for s in spec["srcs"] + spec["deps"] if os.path.exists(s))
+    paths = [_src(e)[0] for e in spec["srcs"]] + spec["deps"]
+    return any(os.path.getmtime(p) > t for p in paths if os.path.exists(p))
 
 
 def _nvcc(args):
@@ -45,16 +60,6 @@ def _nvcc(args):
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc failed: " + " ".join(args[-3:]))
     return r.stderr
-
-
-def build_variant(tag: str, defines) -> str:
-    """Experiment build of libemb with extra -D flags into exp/libemb_<tag>.so (selected at
-    load time with EMB_LIB=<path>; the default library is untouched)."""
-    spec = dict(LIBS["emb"])
-    spec["out"] = os.path.join(PKG, "exp", f"libemb_{tag}.so")
-    os.makedirs(os.path.dirname(spec["out"]), exist_ok=True)
-    _build_one(f"emb_{tag}", spec, True, False, [f"-D{d}" for d in defines])
-    return spec["out"]
 
 
 def build(names=None, force: bool = False, verbose: bool = False) -> None:
@@ -74,9 +79,10 @@ def _build_one(name, spec, force, verbose, extra=()):
         os.makedirs(objdir, exist_ok=True)
         comp = [f for f in FLAGS if f != "-shared"] + list(extra)
         jobs = []
-        for src in spec["srcs"]:
-            obj = os.path.join(objdir, os.path.basename(src) + ".o")
-            jobs.append((obj, [*ARCH, *comp, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]))
+        for entry in spec["srcs"]:
+            src, stem, defs = _src(entry)
+            obj = os.path.join(objdir, stem + ".o")
+            jobs.append((obj, [*ARCH, *comp, *defs, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]))
         with ThreadPoolExecutor(max_workers=min(len(jobs), os.cpu_count() or 4)) as ex:
             logs = list(ex.map(lambda j: _nvcc(j[1]), jobs))
         _nvcc([*ARCH, "-shared", "-Xcompiler", "-fPIC", *[j[0] for j in jobs], "-o", spec["out"] + ".tmp"])

@@ -83,27 +83,27 @@ __device__ __forceinline__ bool wait_flags_geq(const uint32_t* flags, int G, int
   return true;
 }
 
-// VB bytes per lane vector, NV vectors per lane (row = 32*VB*NV bytes when all lanes active)
-// V2: each slice's distinct rows are compacted into a per-warp shared-memory list (row id
+// VB bytes per lane vector, NV vectors per lane (row = 32*VB*NV bytes when all lanes active).
+// Each 32-id slice's distinct rows are compacted into a per-warp shared-memory list (row id
 // and multiplicity in one word) and scattered from it with broadcast LDS.128 reads, 8
-// REDs per iteration -- no SHFL / find-first-set chain per distinct row
+// REDs per iteration -- no SHFL / find-first-set chain per distinct row.
 //
-// HC > 0 (needs V2): each warp privatizes up to HC dW rows of its current chunk in shared
+// HC > 0: each warp privatizes up to HC dW rows of its current chunk in shared
 // memory (direct-mapped by a multiplicative hash of the row id, first come first served,
 // a row whose slot is taken goes straight to L2).  A zipf-hot row then costs one RED per
 // chunk (the flush at the chunk's end) instead of one per bag slice: same-address
 // atomics on the hottest rows are what serialize in the L2.
-template <int VB, int NV, bool V2 = false, int HC = 0>
+template <int VB, int NV, int HC = 0>
 __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__ BwdParams p) {
-  static_assert(HC == 0 || (V2 && HC <= 32 && (HC & (HC - 1)) == 0), "cache: V2, power of two <= 32 slots");
+  static_assert(HC == 0 || (HC <= 32 && (HC & (HC - 1)) == 0), "cache: power of two <= 32 slots");
   constexpr int W = VB / 4;
   const int lane = threadIdx.x & 31;
   const bool active = lane < p.lanes;
   const int64_t rowbytes = (int64_t)p.d * 4;
   const int64_t B = p.B;
   __shared__ __align__(16) uint32_t bwd_ring[kBlock / 32][128];     // per-warp id ring
-  __shared__ __align__(16) uint32_t bwd_list[V2 ? kBlock / 32 : 1][V2 ? 80 : 4];  // V2: compacted (id|mult) + mult
-  const uint32_t list_s = (uint32_t)__cvta_generic_to_shared(&bwd_list[V2 ? (threadIdx.x >> 5) : 0][0]);
+  __shared__ __align__(16) uint32_t bwd_list[kBlock / 32][80];   // compacted (id|mult) + mult
+  const uint32_t list_s = (uint32_t)__cvta_generic_to_shared(&bwd_list[threadIdx.x >> 5][0]);
   // HC: per-warp row cache [HC][32*VB*NV bytes] + tags [HC] in dynamic shared memory
   constexpr uint32_t kRowB = 32u * VB * NV;
   constexpr uint32_t kEmpty = 0xffffffffu;
@@ -215,104 +215,83 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
             asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(ring_s + (uint32_t)(((r0 + lane) & 127) * 4)) : "memory");
           const unsigned same = __match_any_sync(kFull, x);
           const bool lead = (x & 0x80000000u) == 0 && (__ffs(same) - 1) == lane;
-          unsigned leaders = __ballot_sync(kFull, lead);
+          const unsigned leaders = __ballot_sync(kFull, lead);
           // row id and multiplicity travel in one word (ids < 2^26): one SHFL per distinct
           // row instead of two -- the leader loop is bound by the MIO pipe
           const uint32_t xm = pack ? (x | ((uint32_t)__popc(same) << 26)) : x;
-          if constexpr (V2) {
-            const int n = __popc(leaders);
-            if (lead) {
-              const uint32_t at = list_s + 4u * (uint32_t)__popc(leaders & ((1u << lane) - 1u));
-              asm volatile("st.shared.u32 [%0], %1;" ::"r"(at), "r"(xm) : "memory");
-              if (!pack) asm volatile("st.shared.u32 [%0], %1;" ::"r"(at + 160u), "r"((uint32_t)__popc(same)) : "memory");
+          const int n = __popc(leaders);
+          if (lead) {
+            const uint32_t at = list_s + 4u * (uint32_t)__popc(leaders & ((1u << lane) - 1u));
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(at), "r"(xm) : "memory");
+            if (!pack) asm volatile("st.shared.u32 [%0], %1;" ::"r"(at + 160u), "r"((uint32_t)__popc(same)) : "memory");
+          }
+          __syncwarp();
+          for (int k = 0; k < n; k += 8) {
+            uint32_t wv[8], mv[8];
+            asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
+                         : "r"(list_s + 4u * k) : "memory");
+            asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[4]), "=r"(wv[5]), "=r"(wv[6]), "=r"(wv[7])
+                         : "r"(list_s + 4u * k + 16u) : "memory");
+            if (!pack) {
+              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[0]), "=r"(mv[1]), "=r"(mv[2]), "=r"(mv[3])
+                           : "r"(list_s + 4u * k + 160u) : "memory");
+              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[4]), "=r"(mv[5]), "=r"(mv[6]), "=r"(mv[7])
+                           : "r"(list_s + 4u * k + 176u) : "memory");
             }
-            __syncwarp();
-            for (int k = 0; k < n; k += 8) {
-              uint32_t wv[8], mv[8];
-              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
-                           : "r"(list_s + 4u * k) : "memory");
-              asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(wv[4]), "=r"(wv[5]), "=r"(wv[6]), "=r"(wv[7])
-                           : "r"(list_s + 4u * k + 16u) : "memory");
-              if (!pack) {
-                asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[0]), "=r"(mv[1]), "=r"(mv[2]), "=r"(mv[3])
-                             : "r"(list_s + 4u * k + 160u) : "memory");
-                asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(mv[4]), "=r"(mv[5]), "=r"(mv[6]), "=r"(mv[7])
-                             : "r"(list_s + 4u * k + 176u) : "memory");
-              }
 #pragma unroll
-              for (int u = 0; u < 8; ++u) {
-                if constexpr (HC > 0) {
-                  if (k + u < n) {
-                    const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
-                    const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
-                    const uint32_t h = HC == 1 ? 0u : (xl * 2654435761u) >> (32 - kLogHC);
-                    // lane 0 alone reads and claims the tag (no cross-lane access to it); the
-                    // shuffle hands its decision to the warp
-                    uint32_t tg = 0;
-                    if (lane == 0) {
-                      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * h) : "memory");
-                      if (tg == kEmpty) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * h), "r"(xl) : "memory");
-                    }
-                    tg = __shfl_sync(kFull, tg, 0);
-                    const bool hit = tg == xl, claim = tg == kEmpty;
-                    if (active) {
+            for (int u = 0; u < 8; ++u) {
+              if constexpr (HC > 0) {
+                if (k + u < n) {
+                  const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
+                  const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
+                  const uint32_t h = HC == 1 ? 0u : (xl * 2654435761u) >> (32 - kLogHC);
+                  // lane 0 alone reads and claims the tag (no cross-lane access to it); the
+                  // shuffle hands its decision to the warp
+                  uint32_t tg = 0;
+                  if (lane == 0) {
+                    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(tg) : "r"(tag_s + 4u * h) : "memory");
+                    if (tg == kEmpty) asm volatile("st.shared.u32 [%0], %1;" ::"r"(tag_s + 4u * h), "r"(xl) : "memory");
+                  }
+                  tg = __shfl_sync(kFull, tg, 0);
+                  const bool hit = tg == xl, claim = tg == kEmpty;
+                  if (active) {
 #pragma unroll
-                      for (int v = 0; v < NV; ++v) {
-                        uint32_t gm[W];
+                    for (int v = 0; v < NV; ++v) {
+                      uint32_t gm[W];
 #pragma unroll
-                        for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
-                        const uint32_t sa = cache_s + h * kRowB + (uint32_t)(v * 32 + lane) * VB;
-                        if (hit) {                            // this lane's columns only: no atomics
-                          uint32_t cv[W];
-                          lds_bytes<VB>(sa, cv);
+                      for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
+                      const uint32_t sa = cache_s + h * kRowB + (uint32_t)(v * 32 + lane) * VB;
+                      if (hit) {                            // this lane's columns only: no atomics
+                        uint32_t cv[W];
+                        lds_bytes<VB>(sa, cv);
 #pragma unroll
-                          for (int i = 0; i < W; ++i) cv[i] = __float_as_uint(__uint_as_float(cv[i]) + __uint_as_float(gm[i]));
-                          sts_bytes<VB>(sa, cv);
-                        } else if (claim) {
-                          sts_bytes<VB>(sa, gm);
-                        } else {
-                          red_add_vec<VB>(reinterpret_cast<float*>(dwl + (uint64_t)xl * (uint64_t)rowbytes + v * 32 * VB), gm);
-                        }
+                        for (int i = 0; i < W; ++i) cv[i] = __float_as_uint(__uint_as_float(cv[i]) + __uint_as_float(gm[i]));
+                        sts_bytes<VB>(sa, cv);
+                      } else if (claim) {
+                        sts_bytes<VB>(sa, gm);
+                      } else {
+                        red_add_vec<VB>(reinterpret_cast<float*>(dwl + (uint64_t)xl * (uint64_t)rowbytes + v * 32 * VB), gm);
                       }
                     }
                   }
-                  continue;
                 }
-                if (k + u < n && active) {
-                  const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
-                  const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
-                  char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
+                continue;
+              }
+              if (k + u < n && active) {
+                const uint32_t xl = pack ? (wv[u] & 0x03ffffffu) : wv[u];
+                const float m = pack ? (float)(wv[u] >> 26) : (float)mv[u];
+                char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
 #pragma unroll
-                  for (int v = 0; v < NV; ++v) {
-                    uint32_t gm[W];
+                for (int v = 0; v < NV; ++v) {
+                  uint32_t gm[W];
 #pragma unroll
-                    for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
-                    red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), gm);
-                  }
+                  for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
+                  red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), gm);
                 }
               }
             }
-            __syncwarp();                                 // the list is rewritten by the next slice
-            continue;
           }
-          const float mult = (float)__popc(same);
-          while (leaders) {
-            const int l = __ffs(leaders) - 1;
-            leaders &= leaders - 1;
-            const uint32_t v = __shfl_sync(kFull, xm, l);
-            const uint32_t xl = pack ? (v & 0x03ffffffu) : v;
-            const float m = pack ? (float)(v >> 26) : __shfl_sync(kFull, mult, l);
-            if (active) {
-              char* rp = dwl + (uint64_t)xl * (uint64_t)rowbytes;
-#pragma unroll
-              for (int v = 0; v < NV; ++v) {
-                uint32_t gm[W];
-#pragma unroll
-                for (int i = 0; i < W; ++i) gm[i] = __float_as_uint(m == 1.0f ? __uint_as_float(g[v][i]) : m * __uint_as_float(g[v][i]));
-                red_add_vec<VB>(reinterpret_cast<float*>(rp + v * 32 * VB), gm);
-              }
-            }
-          }
+          __syncwarp();                                 // the list is rewritten by the next slice
         }
       }
       asm volatile("cp.async.wait_group 0;" ::: "memory");   // no copy outlives the chunk

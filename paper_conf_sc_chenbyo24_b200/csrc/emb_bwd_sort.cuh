@@ -1,26 +1,24 @@
-// emb_bwd_sort.cuh -- SURVEY row f2, second algorithm ("bwd_algo" = 1): the EMB backward
-// as a transpose of the sparse input (counting sort of the lookups by dW row) followed by
-// a segmented gather-sum, so every distinct dW row receives ONE atomic add per segment of
-// the sorted list instead of one per bag slice.
+// emb_bwd_sort.cuh -- SURVEY row f2, second algorithm (option "bwd_algo" = 1): the EMB
+// backward as a transpose of the sparse input (an LSD radix sort of the lookups by dW row)
+// followed by a segmented gather-sum, so every distinct dW row receives ONE atomic add per
+// run of the sorted list instead of one per bag slice.
 //
 // Same definition as emb_bwd.cuh (§V; adjoint of the sum pooling of
 // L91-95):   dW_t[x, :] += sum over bags (t, b), positions j with x_t[j] = x, of dY[b, t, :]
 //
-// Steps (all stream-ordered on the caller's stream; only step 5 reads peers' memory):
-//   1. hist     cnt[g] = number of lookups of global row g (g = rowbase[t] + x), warp-
-//               aggregated atomics (zipf-hot rows repeat inside a warp's 32 lookups)
-//   2. scan     cnt <- exclusive prefix sum (3 kernels: tile sums, scan of the tile sums,
-//               tile scan + offset)
-//   3. scatter  every lookup (t, b, x) writes {dY row code of (b, t), g} at cnt[g]++ ; the
-//               code is (owning DP rank << 28) | (b - s_dst) * T + t_global
-//   4. (memset of cnt before step 1)
-//   5. reduce   persistent warps claim tasks of S consecutive sorted entries, gather each
+// Steps (all stream-ordered on the caller's stream; only the reduce reads peers' memory):
+//   1. gen      entries in position order: {dY row code of the bag, global row g =
+//               rowbase[t] + x}; the code is (owning DP rank << 28) | (b - s_dst) * T + t
+//   2. sort     per 9-bit digit: upsweep of per-tile digit histograms, the 3-kernel scan
+//               (tile sums, scan of the tile sums, tile scan + offset) over the digit-major
+//               histogram matrix, stable downsweep (3 passes cover 27-bit rows)
+//   3. reduce   persistent warps claim tasks of S consecutive sorted entries, gather each
 //               entry's dY vector (one-sided load from the DP rank's grad slot), sum runs of
 //               equal g in registers and red.add the run into dW_t[x] (two-group software
 //               pipeline of row loads as in the forward); the last CTA releases "done".
-// Order of the fp32 sum inside a run follows the atomic cursor of step 3 (unspecified), so
-// results match the oracle within the order-independent bound and exactly on integer-valued
-// gradients, like the atomic-scatter algorithm.
+// The sort is stable, so a run's fp32 sum follows position order; across runs and warps
+// the atomics make the order unspecified: results match the oracle within the order-
+// independent bound and exactly on integer-valued gradients, like the atomic scatter.
 #pragma once
 
 #include "emb_bwd.cuh"
@@ -53,7 +51,6 @@ struct SortParams {
 };
 
 constexpr int kScanTile = 4096;    // counters per scan tile (256 threads x 16)
-constexpr int kHistSpan = 1024;    // lookups per warp task in hist
 constexpr int kSortTask = 256;     // sorted entries per warp task in reduce
 
 __device__ __forceinline__ int64_t sort_nnz(const SortParams& p) {
@@ -69,50 +66,6 @@ __device__ __forceinline__ int table_of(const int64_t* tb, int T_r, int64_t j) {
     else hi = mid - 1;
   }
   return lo;
-}
-
-// 1. histogram of lookups per global row
-__global__ void __launch_bounds__(kBlock) emb_bsort_hist_kernel(const __grid_constant__ SortParams p) {
-  extern __shared__ __align__(16) int64_t bs_smem[];
-  int64_t* tb = bs_smem;                    // [T_r + 1] table position bounds
-  int64_t* rb = bs_smem + p.T_r + 1;        // [T_r + 1] row bases
-  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) {
-    tb[i] = __ldg(p.offsets + (int64_t)i * p.B);
-    rb[i] = __ldg(p.rowbase + i);
-  }
-  __syncthreads();
-  const int64_t nnz = tb[p.T_r];
-  if (nnz > p.cap) {                         // workspace too small: skip the step (sticky error)
-    if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr(&p.ctrl->err, 0x4u);
-    return;
-  }
-  const int lane = threadIdx.x & 31;
-  const int64_t nw = (int64_t)gridDim.x * (kBlock / 32);
-  constexpr int KB = 8;                                   // index loads in flight per lane
-  for (int64_t task = (int64_t)blockIdx.x * (kBlock / 32) + (threadIdx.x >> 5); task * kHistSpan < nnz; task += nw) {
-    const int64_t j0 = task * kHistSpan, j1 = min(nnz, j0 + kHistSpan);
-    int t = table_of(tb, p.T_r, j0 + lane);
-    for (int64_t jb = j0; jb < j1; jb += 32 * KB) {
-      int64_t x[KB];
-#pragma unroll
-      for (int k = 0; k < KB; ++k) {
-        const int64_t j = jb + 32 * k + lane;
-        x[k] = j < j1 ? ld_stream_i64(p.indices + j) : 0;
-      }
-#pragma unroll
-      for (int k = 0; k < KB; ++k) {
-        const int64_t j = jb + 32 * k + lane;
-        const bool valid = j < j1;
-        uint32_t g = 0xffffffffu;
-        if (valid) {
-          while (j >= tb[t + 1]) ++t;
-          g = (uint32_t)(rb[t] + x[k]);
-        }
-        const unsigned same = __match_any_sync(kFull, g);
-        if (valid && (__ffs(same) - 1) == lane) atomicAdd(p.cnt + g, (uint32_t)__popc(same));
-      }
-    }
-  }
 }
 
 // 2a. per-tile sums
@@ -192,248 +145,6 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_scan_apply_kernel(const __gr
     const uint32_t ex = block_exscan(v[k], sh, &tot);
     if (base + k * kBlock < p.R) p.cnt[base + k * kBlock] = carry + ex;
     carry += tot;
-  }
-}
-
-// 3. scatter every lookup to its row's segment: warp per chunk of consecutive bags of one
-// table; each lane finds its position's bag in the chunk's offsets (shared memory)
-__global__ void __launch_bounds__(kBlock) emb_bsort_scatter_kernel(const __grid_constant__ SortParams p) {
-  __shared__ int64_t ofs[kBlock / 32][33];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t B = p.B, nbags = (int64_t)p.T_r * B;
-  if (nbags == 0) return;
-  const int64_t nnz = sort_nnz(p);
-  if (nnz > p.cap) return;
-  const int64_t cb64 = nnz > 0 ? ((int64_t)p.chunk_rows * nbags + nnz - 1) / nnz : 31;
-  const int cb = (int)(cb64 < 1 ? 1 : (cb64 > 31 ? 31 : cb64));
-  const int64_t cpt = (B + cb - 1) / cb, nchunks = cpt * p.T_r;
-  const int64_t nw = (int64_t)gridDim.x * (kBlock / 32);
-  for (int64_t c = (int64_t)blockIdx.x * (kBlock / 32) + w; c < nchunks; c += nw) {
-    const int t_l = (int)(c / cpt);
-    const int64_t b0 = (c % cpt) * cb;
-    const int nb = (int)min((int64_t)cb, B - b0);
-    if (lane <= nb) ofs[w][lane] = ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane);
-    __syncwarp();
-    const int64_t pos0 = ofs[w][0], pos1 = ofs[w][nb];
-    const int64_t rb = __ldg(p.rowbase + t_l);
-    const int64_t tglob = __ldg(&p.tables[t_l].tglob);
-    constexpr int KB = 4;                                 // batches of 32 lookups in flight
-    for (int64_t jb = pos0; jb < pos1; jb += 32 * KB) {
-      int64_t x[KB];
-#pragma unroll
-      for (int k = 0; k < KB; ++k) {
-        const int64_t j = jb + 32 * k + lane;
-        x[k] = j < pos1 ? ld_stream_i64(p.indices + j) : 0;
-      }
-      uint32_t g[KB], code[KB], at[KB];
-      unsigned same[KB];
-#pragma unroll
-      for (int k = 0; k < KB; ++k) {
-        const int64_t j = jb + 32 * k + lane;
-        const bool valid = j < pos1;
-        g[k] = 0xffffffffu;
-        code[k] = 0;
-        if (valid) {
-          int lo = 0, hi = nb - 1;                  // last bag with start <= j
-          while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (ofs[w][mid] <= j) lo = mid;
-            else hi = mid - 1;
-          }
-          const int64_t b = b0 + lo;
-          int dst = 0;
-          while (b >= p.bstart[dst + 1]) ++dst;
-          code[k] = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
-          g[k] = (uint32_t)(rb + x[k]);
-        }
-        same[k] = __match_any_sync(kFull, g[k]);
-        at[k] = 0;
-        if (valid && (__ffs(same[k]) - 1) == lane) at[k] = atomicAdd(p.cnt + g[k], (uint32_t)__popc(same[k]));
-      }
-#pragma unroll
-      for (int k = 0; k < KB; ++k) {
-        const int64_t j = jb + 32 * k + lane;
-        const int leader = __ffs(same[k]) - 1;
-        const uint32_t a = __shfl_sync(kFull, at[k], leader) + (uint32_t)__popc(same[k] & ((1u << lane) - 1u));
-        if (j < pos1) p.pairs[a] = make_uint2(code[k], g[k]);
-      }
-    }
-    __syncwarp();
-  }
-}
-
-// ---------------------------------------------------------------------------- bwd_algo 2
-// Same sort, but the histogram and the scatter first aggregate a CTA's span of lookups in
-// a shared-memory hash table (open addressing, kHashSlots keys + counts): a zipf-hot row
-// then costs ONE global atomic per span instead of one per 32 lookups (the same-address
-// atomics on hot counters are what serialize bwd_algo 1).  Keys that find no free slot
-// within kHashProbe probes go straight to the global counter.
-constexpr int kHashSlots = 8192;   // smem: keys + counts (+ bases in scatter) per CTA
-constexpr int kHashProbe = 8;
-constexpr int kHashSpan = 4096;    // lookups per CTA task (load factor <= 1/2)
-constexpr uint32_t kHashEmpty = 0xffffffffu;
-
-__device__ __forceinline__ uint32_t hslot(uint32_t k) { return (k * 2654435761u) >> (32 - 13); }
-
-// insert `c` occurrences of key k; returns false if no slot was found (caller goes global)
-__device__ __forceinline__ bool hash_add(uint32_t* hk, uint32_t* hc, uint32_t k, uint32_t c) {
-  uint32_t h = hslot(k);
-#pragma unroll 1
-  for (int i = 0; i < kHashProbe; ++i) {
-    const uint32_t old = atomicCAS(hk + h, kHashEmpty, k);
-    if (old == kHashEmpty || old == k) {
-      atomicAdd(hc + h, c);
-      return true;
-    }
-    h = (h + 1) & (kHashSlots - 1);
-  }
-  return false;
-}
-
-__device__ __forceinline__ int hash_find(const uint32_t* hk, uint32_t k) {
-  uint32_t h = hslot(k);
-#pragma unroll 1
-  for (int i = 0; i < kHashProbe; ++i) {
-    const uint32_t v = hk[h];
-    if (v == k) return (int)h;
-    if (v == kHashEmpty) return -1;
-    h = (h + 1) & (kHashSlots - 1);
-  }
-  return -1;
-}
-
-// 1'. histogram with per-CTA aggregation over spans of kHashSpan consecutive lookups
-__global__ void __launch_bounds__(kBlock) emb_bsort_hist2_kernel(const __grid_constant__ SortParams p) {
-  extern __shared__ __align__(16) uint32_t hs_smem[];
-  uint32_t* hk = hs_smem;
-  uint32_t* hc = hs_smem + kHashSlots;
-  int64_t* tb = reinterpret_cast<int64_t*>(hs_smem + 2 * kHashSlots);
-  int64_t* rb = tb + p.T_r + 1;
-  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) {
-    tb[i] = __ldg(p.offsets + (int64_t)i * p.B);
-    rb[i] = __ldg(p.rowbase + i);
-  }
-  for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
-    hk[i] = kHashEmpty;
-    hc[i] = 0;
-  }
-  __syncthreads();
-  const int64_t nnz = tb[p.T_r];
-  if (nnz > p.cap) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr(&p.ctrl->err, 0x4u);
-    return;
-  }
-  const int lane = threadIdx.x & 31;
-  for (int64_t task = blockIdx.x; task * kHashSpan < nnz; task += gridDim.x) {
-    const int64_t j0 = task * kHashSpan, j1 = min(nnz, j0 + kHashSpan);
-    constexpr int KB = kHashSpan / kBlock;               // 16 lookups per thread
-    int64_t x[KB];
-#pragma unroll
-    for (int k = 0; k < KB; ++k) {
-      const int64_t j = j0 + (int64_t)k * kBlock + threadIdx.x;
-      x[k] = j < j1 ? ld_stream_i64(p.indices + j) : 0;
-    }
-    int t = table_of(tb, p.T_r, j0 + threadIdx.x);
-#pragma unroll
-    for (int k = 0; k < KB; ++k) {
-      const int64_t j = j0 + (int64_t)k * kBlock + threadIdx.x;
-      const bool valid = j < j1;
-      uint32_t g = kHashEmpty;
-      if (valid) {
-        while (j >= tb[t + 1]) ++t;
-        g = (uint32_t)(rb[t] + x[k]);
-      }
-      const unsigned same = __match_any_sync(kFull, g);
-      if (valid && (__ffs(same) - 1) == lane && !hash_add(hk, hc, g, (uint32_t)__popc(same)))
-        atomicAdd(p.cnt + g, (uint32_t)__popc(same));
-    }
-    __syncthreads();
-    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {   // flush + clear
-      const uint32_t k = hk[i];
-      if (k != kHashEmpty) {
-        atomicAdd(p.cnt + k, hc[i]);
-        hk[i] = kHashEmpty;
-        hc[i] = 0;
-      }
-    }
-    __syncthreads();
-  }
-}
-
-// 3'. scatter with per-CTA aggregation: CTA task = a chunk of consecutive bags of one table
-// (<= 1024 bags, ~kHashSpan lookups).  Pass 1 counts the chunk's keys in the hash table,
-// then one returning global atomic per distinct key reserves its run, pass 2 hands out
-// positions inside the runs with shared-memory atomics.
-__global__ void __launch_bounds__(kBlock) emb_bsort_scatter2_kernel(const __grid_constant__ SortParams p) {
-  constexpr int kMaxCB = 1024;
-  extern __shared__ __align__(16) uint32_t hs_smem[];
-  uint32_t* hk = hs_smem;
-  uint32_t* hc = hs_smem + kHashSlots;                    // counts, then local cursors
-  uint32_t* hb = hs_smem + 2 * kHashSlots;                // reserved global base per key
-  int64_t* ofs = reinterpret_cast<int64_t*>(hs_smem + 3 * kHashSlots);   // [kMaxCB + 1]
-  const int64_t B = p.B, nbags = (int64_t)p.T_r * B;
-  if (nbags == 0) return;
-  const int64_t nnz = sort_nnz(p);
-  if (nnz > p.cap) return;
-  for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
-    hk[i] = kHashEmpty;
-    hc[i] = 0;
-  }
-  const int64_t cb64 = nnz > 0 ? ((int64_t)kHashSpan * nbags + nnz - 1) / nnz : kMaxCB;
-  const int cb = (int)(cb64 < 1 ? 1 : (cb64 > kMaxCB ? kMaxCB : cb64));
-  const int64_t cpt = (B + cb - 1) / cb, nchunks = cpt * p.T_r;
-  __syncthreads();
-  for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
-    const int t_l = (int)(c / cpt);
-    const int64_t b0 = (c % cpt) * cb;
-    const int nb = (int)min((int64_t)cb, B - b0);
-    for (int i = threadIdx.x; i <= nb; i += blockDim.x) ofs[i] = ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + i);
-    __syncthreads();
-    const int64_t pos0 = ofs[0], pos1 = ofs[nb];
-    const int64_t rb = __ldg(p.rowbase + t_l);
-    const int64_t tglob = __ldg(&p.tables[t_l].tglob);
-    // pass 1: counts
-    for (int64_t j = pos0 + threadIdx.x; j - threadIdx.x < pos1; j += kBlock) {
-      const bool valid = j < pos1;
-      const uint32_t g = valid ? (uint32_t)(rb + ld_stream_i64(p.indices + j)) : kHashEmpty;
-      const unsigned same = __match_any_sync(kFull, g);
-      if (valid && (__ffs(same) - 1) == (int)(threadIdx.x & 31)) hash_add(hk, hc, g, (uint32_t)__popc(same));
-    }
-    __syncthreads();
-    // reserve each key's run: one returning global atomic per distinct key
-    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
-      const uint32_t k = hk[i];
-      if (k != kHashEmpty) {
-        hb[i] = atomicAdd(p.cnt + k, hc[i]);
-        hc[i] = 0;
-      }
-    }
-    __syncthreads();
-    // pass 2: positions
-    for (int64_t j = pos0 + threadIdx.x; j - threadIdx.x < pos1; j += kBlock) {
-      if (j < pos1) {
-        const uint32_t g = (uint32_t)(rb + ld_stream_i64(p.indices + j));
-        int lo = 0, hi = nb - 1;                          // last bag with start <= j
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (ofs[mid] <= j) lo = mid;
-          else hi = mid - 1;
-        }
-        const int64_t b = b0 + lo;
-        int dst = 0;
-        while (b >= p.bstart[dst + 1]) ++dst;
-        const uint32_t code = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
-        const int h = hash_find(hk, g);
-        const uint32_t at = h >= 0 ? hb[h] + atomicAdd(hc + h, 1u) : atomicAdd(p.cnt + g, 1u);
-        p.pairs[at] = make_uint2(code, g);
-      }
-    }
-    __syncthreads();
-    for (int i = threadIdx.x; i < kHashSlots; i += blockDim.x) {
-      hk[i] = kHashEmpty;
-      hc[i] = 0;
-    }
-    __syncthreads();
   }
 }
 

@@ -33,6 +33,11 @@ using namespace emb;
 namespace {
 
 constexpr uint64_t kMagic = 0x454d42504741531full;  // "EMBPGAS"
+// Output ring depth.  Peer p's forward e+3 writes into slot e % 3 of this rank only after
+// p's forward e+2 acquired this rank's epoch-(e+2) signal, i.e. after this rank launched
+// its forward e+2: so Y_r(e) stays intact until this rank's second subsequent forward, and
+// the host path can overlap the D2H of Y_r(e) with forward e+1.
+constexpr int kOutSlots = 3;
 
 struct PeerBlob {
   uint64_t magic;
@@ -96,7 +101,7 @@ struct emb_ctx {
   Ctrl* ctrl = nullptr;
   uint64_t epoch = 0;
   // options
-  int chunk_rows = 0, ctas_per_sm = 0, stagger = 1, unroll = 0, minblocks = 0, sidx = 1, carveout = 0, ds = 0;  // 0: auto per tile
+  int chunk_rows = 0, ctas_per_sm = 0, stagger = 1, carveout = 0;  // 0: auto per tile
   int64_t timeout_ns = 10000000000ll;
   // gather tiling
   int lanes = 32, vb = 16, nv = 1;
@@ -108,13 +113,16 @@ struct emb_ctx {
   int64_t* d_idx_stage = nullptr;
   size_t idx_cap = 0;
   // pipelined host path: two input stages, copy-in / copy-out streams, events
-  int64_t* p_off[2] = {nullptr, nullptr};
-  int64_t* p_idx[2] = {nullptr, nullptr};
-  size_t p_cap[2] = {0, 0};
+  char* p_off[2] = {nullptr, nullptr};
+  char* p_idx[2] = {nullptr, nullptr};
+  size_t p_cap[2] = {0, 0};               // bytes of p_idx[k]
+  size_t p_offcap[2] = {0, 0};            // bytes of p_off[k]
   cudaStream_t s_in = nullptr, s_out = nullptr;
-  cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
-  bool kern_rec[2] = {false, false}, out_rec[2] = {false, false};
+  cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr};
+  cudaEvent_t ev_out[kOutSlots] = {nullptr, nullptr, nullptr};   // D2H of the output of epoch e, by e % kOutSlots
+  bool kern_rec[2] = {false, false}, out_rec[kOutSlots] = {false, false, false};
   uint64_t host_calls = 0;
+  bool wait_pending = false;            // last forward used EMB_FWD_SEPARATE_WAIT and emb_wait is due
   // f2 backward
   bool bwd_enabled = false;
   size_t grad_off = 0, gslot_bytes = 0;
@@ -122,25 +130,22 @@ struct emb_ctx {
   uint64_t bepoch = 0;
   bool bwd_ready_pending = false;
   int bwd_interleave = 1;
-  int bwd_v2 = 1;                  // backward slice scatter from a compacted smem list
-  int bwd_cache = 16;              // per-warp dW row cache slots (0 off; 8 / 16 / 32; needs bwd_v2)
-  int bwd_chunk_rows = 0;          // backward chunk target rows (0: chunk_rows)
+  int bwd_cache = 16;              // per-warp dW row cache slots (0 off, 16 on; one vector per lane)
+  int bwd_chunk_rows = 0;          // backward chunk target rows (0: chunk_rows, else 256)
   int bwd_group = 8;               // tables interleaved at a time in the backward (0: all T_r)
-  int bwd_algo = 0;                // 0: atomic scatter per bag slice; 1: counting sort + segmented sum
-  int64_t bs_cap = 0, bs_R = 0, bs_nblk = 0;   // bwd_algo 1 workspace
+  int bwd_algo = 0;                // 0: atomic scatter per bag slice; 1: radix sort + segmented sum
+  int64_t bs_cap = 0, bs_R = 0;    // bwd_algo 1 workspace: entries, local rows
   int64_t* d_rowbase = nullptr;
-  uint32_t* d_bcnt = nullptr;
-  uint32_t* d_bsum = nullptr;
   uint2* d_pairs = nullptr;
-  uint2* d_pairs_b = nullptr;      // bwd_algo 3: radix-sort ping-pong buffer
-  uint32_t* d_ghist = nullptr;     // bwd_algo 3: [256][tiles] digit histograms
+  uint2* d_pairs_b = nullptr;      // radix-sort ping-pong buffer
+  uint32_t* d_ghist = nullptr;     // [512][tiles] digit histograms
   uint32_t* d_rbsum = nullptr;
   int64_t rs_nblk = 0;
   int fwd_interleave = 0;
-  int row_l2 = 0, out_l2 = 0;      // experiment builds (EMB_EXP_L2) only
   int tail_div = 4;                // guided tail of the forward's chunk schedule
+  int64_t d2h_delay_us = 0;        // test hook: stall the host path's copy-out stream before each D2H
   int tma_store = 0;          // f4: stage pooled vectors, ship 4 per TMA scatter4
-  void* d_tmaps = nullptr;    // f4: CUtensorMap [2 slots][kMaxG] of every rank's output slots
+  void* d_tmaps = nullptr;    // f4: CUtensorMap [kOutSlots][kMaxG] of every rank's output slots
   float** d_dW = nullptr;
   std::vector<void*> h_dW;
   int blanes = 32, bvb = 16, bnv = 1;
@@ -167,55 +172,30 @@ struct emb_ctx {
   } while (0)
 
 static size_t esize(emb_dtype_t t) { return t == EMB_F32 ? 4 : 2; }
-// register budget per tile: one vector per lane fits 64 registers (4 CTAs of 256 per SM,
-// no spills for any dtype pair); fp32 rows of 16-B lanes take 48 registers (5 CTAs, 40
-// warps/SM: zipf weak 0.70 -> 0.67 ms, strong 6.66 -> 6.39 ms; uniform +0.4 %; bf16 rows
-// spill at 48 and stay at 4); wider rows keep the unconstrained build
-static int eff_minblocks(const emb_ctx* c) {
-  if (c->minblocks) return c->minblocks;
-  if (c->nv != 1) return 1;
-  return (c->vb == 16 && c->wdt == EMB_F32) ? 5 : 4;
-}
-// rows per pipeline group: 4 rows for both 8- and 16-byte lane vectors (measured best)
-static int eff_unroll(const emb_ctx* c) { return c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4); }
 // a row exactly covers the warp's 32 lane vectors (lets the row stride be a constant)
 static bool full_row(const emb_ctx* c) { return c->lanes == 32 && (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb * c->nv; }
-// the SIDX id ring (4 x 32 32-bit ids per warp in shared memory, LDS.128 broadcast of 4 ids
-// per row group) is on by default where the kernel has it: full-row tiles with one vector
-// per lane, no bounds check, no row shards, direct stores, 4-row groups (or 2 with 8-B lanes)
-static bool sidx_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
-  const int u = c->unroll ? c->unroll : (c->vb == 8 ? 2 : 4);
-  const int mb = eff_minblocks(c);
-  return c->sidx != 0 && c->nv == 1 && c->lanes == 32 && !check && !shard && !tmast &&
-         (int64_t)c->d * (int64_t)esize(c->wdt) == 32LL * c->vb && ((u == 4 && (mb == 4 || mb == 5 || mb == 6)) || u == 2 || u == 3);
+// fused-kernel variant: f4 TMA stores, per-id validity (f3 row shards / bounds check), or the
+// default direct-store kernel
+static int fwd_mode(bool check, bool shard, bool tmast) {
+  if (check || shard) return kModeFilt;
+  return tmast ? kModeTma : kModeDirect;
 }
-// dual-stream kernel (emb_fwd_ds_kernel): 256-B rows, default options, no bounds check,
-// no row shards, direct stores
-static bool ds_on(const emb_ctx* c, bool check, bool shard, bool tmast) {
-  return c->ds != 0 && c->unroll == 0 && c->minblocks == 0 && !check && !shard && !tmast &&
-         (int64_t)c->d * (int64_t)esize(c->wdt) == 256;
-}
-static KernelFn pick_ds(emb_dtype_t w, emb_dtype_t o, int mb) {
-  if (w == EMB_F32) return o == EMB_F32 ? pick_ds_f32_f32(mb) : pick_ds_f32_bf16(mb);
-  return o == EMB_F32 ? pick_ds_bf16_f32(mb) : pick_ds_bf16_bf16(mb);
-}
-// shared-memory ring of the cp.async pipeline: 8 warps x `unroll` row slots
-static size_t dyn_smem(const emb_ctx* c, bool sidx = false) {
-  if (eff_unroll(c) < 0 && c->nv == 1 && full_row(c) && !c->has_shard)  // ring v2: R rows of 512 B per warp
-    return (size_t)(kBlock / 32) * (size_t)(-eff_unroll(c) == 4 ? 8 : -eff_unroll(c)) * 32 * c->vb;
-  if (eff_unroll(c) >= 8 && c->nv == 1) return (size_t)(kBlock / 32) * eff_unroll(c) * 32 * c->vb;
-  if (sidx) return (size_t)(kBlock / 32) * EMB_SIDX_RING * 128;   // id ring: EMB_SIDX_RING x 32 x 4 B per warp
-  return 0;
+// dynamic shared memory: the per-warp id ring (+ f4: two staging buffers of 4 output rows per warp)
+static size_t fwd_smem(const emb_ctx* c, int mode) {
+  size_t s = (size_t)(kBlock / 32) * kSidxWarpBytes;
+  if (mode == kModeTma) s += (size_t)(kBlock / 32) * 8 * (size_t)c->d * esize(c->odt);
+  return mode == kModeFilt ? 0 : s;
 }
 
 // ---------------------------------------------------------------------------- kernel dispatch
 namespace {
 
-KernelFn pick_kernel(emb_dtype_t w, emb_dtype_t o, int vb, int nv, int unroll, bool check, int mb, bool full, bool sidx, bool shard = false, bool tmast = false) {
-  if (w == EMB_F32 && o == EMB_F32) return pick_tile_f32_f32(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
-  if (w == EMB_F32 && o == EMB_BF16) return pick_tile_f32_bf16(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
-  if (w == EMB_BF16 && o == EMB_F32) return pick_tile_bf16_f32(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
-  return pick_tile_bf16_bf16(vb, nv, unroll, check, mb, full, sidx, shard, tmast);
+KernelFn pick_kernel(const emb_ctx* c, int mode) {
+  const bool full = full_row(c);
+  if (c->wdt == EMB_F32 && c->odt == EMB_F32) return pick_fwd_f32_f32(c->vb, c->nv, full, mode);
+  if (c->wdt == EMB_F32 && c->odt == EMB_BF16) return pick_fwd_f32_bf16(c->vb, c->nv, full, mode);
+  if (c->wdt == EMB_BF16 && c->odt == EMB_F32) return pick_fwd_bf16_f32(c->vb, c->nv, full, mode);
+  return pick_fwd_bf16_bf16(c->vb, c->nv, full, mode);
 }
 
 // row-gather tiling: VB bytes per lane-vector, NV vectors per lane, `lanes` active lanes
@@ -357,6 +337,7 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     if (((uintptr_t)w) % 16 != 0) FAIL(c, EMB_ERR_ARG, "local_weights[%d] not 16-byte aligned", i);
     td[i].w = w;
     td[i].rows = lsh[i].hi - lsh[i].lo;
+    td[i].mrows = rows[lsh[i].t];
     td[i].tglob = lsh[i].t;
     td[i].part = lsh[i].part;
     td[i].lo = lsh[i].lo;
@@ -388,12 +369,12 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     CK(c, cudaMemcpy(c->d_unpack_base, base.data(), num_tables * sizeof(int64_t), cudaMemcpyHostToDevice));
     CK(c, cudaMemcpy(c->d_unpack_stride, stride.data(), num_tables * sizeof(int32_t), cudaMemcpyHostToDevice));
   }
-  // symmetric buffer: [flags: G u32, padded to 512 B][slot 0][slot 1]
+  // symmetric buffer: [flags: G u32, padded to 512 B][output slot 0][slot 1][slot 2]
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   // header: [fwd flags G u32 @0][bwd ready G u32 @64][bwd done G u32 @128], 512 B
   c->slot_off = 512;
   c->slot_bytes = round_up((size_t)Br * (size_t)num_tables * (size_t)dim * osz, 512);
-  c->sym_bytes = c->slot_off + 2 * c->slot_bytes;
+  c->sym_bytes = c->slot_off + kOutSlots * c->slot_bytes;
   if (c->has_shard) {  // f3 partial slots [2][B_r][T_sh * S_max][d] fp32
     if (dim % 4 != 0) FAIL(c, EMB_ERR_ARG, "row-sharded tables need dim %% 4 == 0");
     c->part_off = c->sym_bytes;
@@ -484,18 +465,12 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
   // the in-kernel peer wait of another rank sharing this GPU).
   {
     cudaFuncAttributes a;
-    const bool full = full_row(c);
-    for (int chk = 0; chk < 2; ++chk) {
-      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
-                                            full, sidx_on(c, chk != 0, c->has_shard && chk == 0, false),
-                                            c->has_shard && chk == 0));
-      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
-                                            full, sidx_on(c, chk != 0, false, false), false));
-      cudaFuncGetAttributes(&a, pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk != 0, eff_minblocks(c),
-                                            full, false, false));
+    for (int mode : {kModeDirect, kModeFilt, kModeTma}) {
+      KernelFn k = pick_kernel(c, mode);
+      if (k) cudaFuncGetAttributes(&a, k);
     }
-    if (c->d * (int64_t)esize(c->wdt) == 256) cudaFuncGetAttributes(&a, pick_ds(c->wdt, c->odt, c->ds));
     cudaFuncGetAttributes(&a, emb_wait_kernel);
+    cudaFuncGetAttributes(&a, emb_sleep_kernel);
     cudaFuncGetAttributes(&a, emb_unpack_kernel);
     cudaFuncGetAttributes(&a, emb_unpack8_kernel);
     cudaFuncGetAttributes(&a, emb_combine_kernel<float>);
@@ -506,30 +481,18 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2>);
     cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 2, true>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 4, true>);
-    cudaFuncGetAttributes(&a, emb_bsort_hist_kernel);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, 16>);
+    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, 16>);
     cudaFuncGetAttributes(&a, emb_bsort_scan_sum_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scan_top_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_scan_apply_kernel);
-    cudaFuncGetAttributes(&a, emb_bsort_scatter_kernel);
-    cudaFuncGetAttributes(&a, emb_bsort_hist2_kernel);
     cudaFuncGetAttributes(&a, emb_bradix_gen_kernel);
     cudaFuncGetAttributes(&a, emb_bradix_up_kernel);
     cudaFuncGetAttributes(&a, emb_bradix_down_kernel);
-    cudaFuncGetAttributes(&a, emb_bsort_scatter2_kernel);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2>);
     cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 4>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 8>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 16>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<8, 1, true, 32>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 8>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 16>);
-    cudaFuncGetAttributes(&a, emb_bwd_kernel<16, 1, true, 32>);
     cudaGetLastError();
   }
   return EMB_OK;
@@ -555,11 +518,15 @@ emb_status_t emb_register_sharded_tables(emb_ctx_t* c, int32_t num_tables, const
                        global_batch, local_weights);
 }
 
+static char* out_slot(emb_ctx_t* c, int g, uint64_t epoch) {   // rank g's output slot of `epoch`
+  return c->peer_base[g] + c->peer_slot_off[g] + (size_t)(epoch % kOutSlots) * c->peer_slot_bytes[g];
+}
+
 static emb_status_t launch_combine(emb_ctx_t* c, cudaStream_t s) {
   if (!c->has_shard) return EMB_OK;
-  const int slot = (int)(c->epoch & 1);
-  const float* part = reinterpret_cast<const float*>(c->sym + c->part_off + (size_t)slot * c->pslot_bytes);
-  char* out = c->sym + c->slot_off + (size_t)slot * c->slot_bytes;
+  const int pslot = (int)(c->epoch & 1);
+  const float* part = reinterpret_cast<const float*>(c->sym + c->part_off + (size_t)pslot * c->pslot_bytes);
+  char* out = out_slot(c, c->rank, c->epoch);
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   const int64_t total = Br * c->T_sh * (c->d / 4);
   int grid = (int)std::min<int64_t>((total + kBlock - 1) / kBlock, (int64_t)c->num_sms * 8);
@@ -585,12 +552,12 @@ static emb_status_t build_tmaps(emb_ctx_t* c) {
   CK(c, cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
   if (!fn || q != cudaDriverEntryPointSuccess) FAIL(c, EMB_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
   auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  std::vector<CUtensorMap> maps(2 * kMaxG);
+  std::vector<CUtensorMap> maps(kOutSlots * kMaxG);
   memset(maps.data(), 0, maps.size() * sizeof(CUtensorMap));
   const size_t eo = esize(c->odt);
-  for (int slot = 0; slot < 2; ++slot)
+  for (int slot = 0; slot < kOutSlots; ++slot)
     for (int g = 0; g < c->G; ++g) {
-      void* base = c->peer_base[g] + c->peer_slot_off[g] + (size_t)slot * c->peer_slot_bytes[g];
+      void* base = out_slot(c, g, (uint64_t)slot);
       const cuuint64_t rows = (cuuint64_t)(c->bstart[g + 1] - c->bstart[g]) * (cuuint64_t)c->T;
       cuuint64_t dims[2] = {(cuuint64_t)c->d, rows};
       cuuint64_t strides[1] = {(cuuint64_t)c->d * eo};
@@ -607,12 +574,13 @@ static emb_status_t build_tmaps(emb_ctx_t* c) {
   return EMB_OK;
 }
 
-static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, bool pgas, char* send,
+static emb_status_t fill_params(emb_ctx_t* c, const void* offsets, const void* indices, bool i32, bool pgas, char* send,
                                 FwdParams* p) {
   memset(p, 0, sizeof(*p));
   p->tables = c->d_tables;
   p->offsets = offsets;
   p->indices = indices;
+  p->idx32 = i32 ? 1 : 0;
   p->B = c->B;
   p->T_r = c->T_r;
   p->d = c->d;
@@ -625,9 +593,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   p->chunk_rows = c->chunk_rows ? c->chunk_rows : (c->wdt == EMB_F32 ? 192 : 256);
   p->stagger = c->stagger;
   p->interleave = c->fwd_interleave;
-  p->row_l2 = c->row_l2;
   p->tail_div = c->tail_div;
-  p->out_l2 = c->out_l2;
   p->ctrl = c->ctrl;
   p->timeout_ns = c->timeout_ns;
   for (int g = 0; g <= c->G; ++g) p->bstart[g] = c->bstart[g];
@@ -635,19 +601,20 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   p->my_flags = reinterpret_cast<const uint32_t*>(c->sym);
   const size_t osz = esize(c->odt);
   if (pgas) {
-    const int slot = (int)(c->epoch & 1);  // epoch already advanced for this forward
+    const int pslot = (int)(c->epoch & 1);  // epoch already advanced for this forward
     p->rowstride = c->T;
     p->use_tglob = 1;
     p->signal = 1;
     for (int g = 0; g < c->G; ++g) {
-      p->out_base[g] = c->peer_base[g] + c->peer_slot_off[g] + (size_t)slot * c->peer_slot_bytes[g];
+      p->out_base[g] = out_slot(c, g, c->epoch);
       p->peer_flag[g] = (g == c->rank) ? nullptr : reinterpret_cast<uint32_t*>(c->peer_base[g]) + c->rank;
       if (c->has_shard)
-        p->part_base[g] = c->peer_base[g] + c->peer_part_off[g] + (size_t)slot * c->peer_pslot_bytes[g];
+        p->part_base[g] = c->peer_base[g] + c->peer_part_off[g] + (size_t)pslot * c->peer_pslot_bytes[g];
     }
     p->part_stride = (int64_t)c->T_sh * c->S_max;
-    p->tmaps = (c->tma_store && c->d_tmaps) ? static_cast<const char*>(c->d_tmaps) + (size_t)slot * kMaxG * sizeof(CUtensorMap)
-                                            : nullptr;
+    p->tmaps = (c->tma_store && c->d_tmaps)
+                   ? static_cast<const char*>(c->d_tmaps) + (size_t)(c->epoch % kOutSlots) * kMaxG * sizeof(CUtensorMap)
+                   : nullptr;
   } else {
     p->rowstride = c->T_r;
     p->use_tglob = 0;
@@ -661,25 +628,29 @@ static emb_status_t fill_params(emb_ctx_t* c, const int64_t* offsets, const int6
   return EMB_OK;
 }
 
+// CTAs of 256 threads the kernel's registers allow per SM (the occupancy it was built for)
+static int ctas_by_regs(KernelFn k) {
+  cudaFuncAttributes a;
+  if (cudaFuncGetAttributes(&a, k) != cudaSuccess || a.numRegs <= 0) return 4;
+  const int per_warp = (int)round_up((size_t)a.numRegs * 32, 256);
+  return std::max(1, 65536 / (per_warp * (kBlock / 32)));
+}
+
 static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags, cudaStream_t s) {
   const bool chk = (flags & EMB_FWD_CHECK_BOUNDS) != 0, shard = p.part_stride > 0, tmast = p.tmaps != nullptr;
-  const bool sx = sidx_on(c, chk, shard, tmast);
-  const bool ds = ds_on(c, chk, shard, tmast);
-  KernelFn k = ds ? pick_ds(c->wdt, c->odt, c->ds)
-                  : pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), chk, eff_minblocks(c), full_row(c), sx, shard, tmast);
-  size_t smem = ds ? (size_t)(kBlock / 32) * 1024 : dyn_smem(c, sx);   // ds: two 512-B id rings per warp
-  if (p.tmaps) smem = std::max(smem, (size_t)(kBlock / 32) * 8 * c->d * esize(c->odt));  // f4 staging (2 x 4 rows)
+  const int mode = fwd_mode(chk, shard, tmast);
+  KernelFn k = pick_kernel(c, mode);
+  if (!k) FAIL(c, EMB_ERR_ARG, "no kernel for this row tiling / mode");
+  const size_t smem = fwd_smem(c, mode);
   if (smem > 0) CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // the gather lives off L1 hits of zipf-hot rows: ask for the smallest shared-memory
-  // carve-out that fits (the rest of the 256 KB per SM becomes L1)
-  // (only without dynamic shared memory: a 0 % carve-out would cap residency at 1 CTA/SM)
-  if (c->carveout >= 0 && smem == 0)
+  // carve-out that still fits the occupancy target (the CTAs the registers allow, each
+  // with its id ring + 1 KB driver reserve), so the rest of the 256 KB per SM stays L1
+  if (c->carveout > 0) {
     CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, c->carveout));
-  // small rings (the SIDX id ring): the smallest carve-out that still fits the occupancy
-  // target (4 CTAs of smem + 1 KB driver reserve each), so the rest stays L1
-  if (c->carveout == 0 && smem > 0 && smem <= 8192) {
-    const size_t want = (size_t)std::max(4, eff_minblocks(c));   // occupancy target (CTAs/SM)
-    const int pct = (int)std::min<size_t>(100, (want * (smem + 1024) * 100 + 233471) / 233472);
+  } else if (c->carveout == 0) {
+    const size_t want = (size_t)ctas_by_regs(k);
+    const int pct = smem == 0 ? 0 : (int)std::min<size_t>(100, (want * (smem + 1024) * 100 + 233471) / 233472);
     CK(c, cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
   }
   int per_sm = c->ctas_per_sm;
@@ -693,42 +664,65 @@ static emb_status_t launch_fwd(emb_ctx_t* c, const FwdParams& p, uint32_t flags,
   return EMB_OK;
 }
 
-emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags, void* stream,
-                         void** out) {
+static emb_status_t wait_impl(emb_ctx_t* c, cudaStream_t s) {
+  c->wait_pending = false;
+  if (c->G > 1) {
+    emb_wait_kernel<<<1, 32, 0, s>>>(c->last);
+    CK(c, cudaGetLastError());
+  }
+  return launch_combine(c, s);
+}
+
+static emb_status_t forward_impl(emb_ctx_t* c, const void* offsets, const void* indices, bool i32, uint32_t flags,
+                                 cudaStream_t s, void** out) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward before emb_register_tables");
   if (c->T_r > 0 && (!offsets || !indices)) FAIL(c, EMB_ERR_ARG, "offsets/indices NULL");
+  if (flags & ~(EMB_FWD_CHECK_BOUNDS | EMB_FWD_SEPARATE_WAIT)) FAIL(c, EMB_ERR_ARG, "unknown flag bits 0x%x", flags);
   CK(c, cudaSetDevice(c->dev));
-  if (c->has_shard && (flags & EMB_FWD_CHECK_BOUNDS))
-    FAIL(c, EMB_ERR_ARG, "EMB_FWD_CHECK_BOUNDS is not supported with row-sharded tables");
   if (c->tma_store) {
     emb_status_t st0 = build_tmaps(c);
     if (st0 != EMB_OK) return st0;
   }
+  // a previous EMB_FWD_SEPARATE_WAIT forward that was never completed is completed first:
+  // the output ring's reuse argument needs every forward's wait before the next launch
+  if (c->wait_pending) {
+    emb_status_t st0 = wait_impl(c, s);
+    if (st0 != EMB_OK) return st0;
+  }
   c->epoch += 1;
   FwdParams p;
-  fill_params(c, offsets, indices, true, nullptr, &p);
+  fill_params(c, offsets, indices, i32, true, nullptr, &p);
   p.wait = (flags & EMB_FWD_SEPARATE_WAIT) ? 0 : 1;
+  p.check = (flags & EMB_FWD_CHECK_BOUNDS) ? 1 : 0;
   c->last = p;
-  emb_status_t st = launch_fwd(c, p, flags, (cudaStream_t)stream);
+  emb_status_t st = launch_fwd(c, p, flags, s);
   if (st != EMB_OK) return st;
   if (!(flags & EMB_FWD_SEPARATE_WAIT)) {  // f3: partials landed (in-kernel wait) -> combine
-    st = launch_combine(c, (cudaStream_t)stream);
+    st = launch_combine(c, s);
     if (st != EMB_OK) return st;
+  } else {
+    c->wait_pending = true;
   }
-  if (out) *out = c->sym + c->slot_off + (size_t)(c->epoch & 1) * c->slot_bytes;
+  if (out) *out = out_slot(c, c->rank, c->epoch);
   return EMB_OK;
+}
+
+emb_status_t emb_forward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags, void* stream,
+                         void** out) {
+  return forward_impl(c, offsets, indices, false, flags, (cudaStream_t)stream, out);
+}
+
+emb_status_t emb_forward_i32(emb_ctx_t* c, const int32_t* offsets, const int32_t* indices, uint32_t flags, void* stream,
+                             void** out) {
+  return forward_impl(c, offsets, indices, true, flags, (cudaStream_t)stream, out);
 }
 
 emb_status_t emb_wait(emb_ctx_t* c, void* stream) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered || c->epoch == 0) FAIL(c, EMB_ERR_STATE, "emb_wait without a forward");
   CK(c, cudaSetDevice(c->dev));
-  if (c->G > 1) {
-    emb_wait_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(c->last);
-    CK(c, cudaGetLastError());
-  }
-  return launch_combine(c, (cudaStream_t)stream);
+  return wait_impl(c, (cudaStream_t)stream);
 }
 
 emb_status_t emb_forward_host(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
@@ -751,74 +745,83 @@ emb_status_t emb_forward_host(emb_ctx_t* c, const int64_t* h_offsets, const int6
   CK(c, cudaMemcpyAsync(c->d_off_stage, h_offsets, noff * sizeof(int64_t), cudaMemcpyHostToDevice, s));
   if (nnz > 0) CK(c, cudaMemcpyAsync(c->d_idx_stage, h_indices, (size_t)nnz * sizeof(int64_t), cudaMemcpyHostToDevice, s));
   void* dout = nullptr;
-  emb_status_t st = emb_forward(c, c->d_off_stage, c->d_idx_stage, flags, stream, &dout);
+  emb_status_t st = forward_impl(c, c->d_off_stage, c->d_idx_stage, false, flags & ~EMB_FWD_SEPARATE_WAIT, s, &dout);
   if (st != EMB_OK) return st;
-  if (flags & EMB_FWD_SEPARATE_WAIT) {
-    st = emb_wait(c, stream);
-    if (st != EMB_OK) return st;
-  }
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   CK(c, cudaMemcpyAsync(h_out, dout, (size_t)Br * c->T * c->d * esize(c->odt), cudaMemcpyDeviceToHost, s));
   return EMB_OK;
 }
 
-emb_status_t emb_forward_host_async(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
-                                    void* stream, void* h_out) {
+// pipelined host path (both index widths): H2D of call k into stage k & 1 on the copy-in
+// stream, the forward on the caller's stream, D2H of Y_r on the copy-out stream
+static emb_status_t host_async_impl(emb_ctx_t* c, const void* h_offsets, const void* h_indices, bool i32,
+                                    uint32_t flags, cudaStream_t s, void* h_out) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_forward_host_async before emb_register_tables");
   if (!h_offsets || !h_out || (c->T_r > 0 && !h_indices)) FAIL(c, EMB_ERR_ARG, "NULL host buffer");
   CK(c, cudaSetDevice(c->dev));
-  cudaStream_t s = (cudaStream_t)stream;
   if (!c->s_in) {
     CK(c, cudaStreamCreateWithFlags(&c->s_in, cudaStreamNonBlocking));
     CK(c, cudaStreamCreateWithFlags(&c->s_out, cudaStreamNonBlocking));
     for (int i = 0; i < 2; ++i) {
       CK(c, cudaEventCreateWithFlags(&c->ev_in[i], cudaEventDisableTiming));
       CK(c, cudaEventCreateWithFlags(&c->ev_kern[i], cudaEventDisableTiming));
-      CK(c, cudaEventCreateWithFlags(&c->ev_out[i], cudaEventDisableTiming));
     }
+    for (int i = 0; i < kOutSlots; ++i) CK(c, cudaEventCreateWithFlags(&c->ev_out[i], cudaEventDisableTiming));
   }
+  const size_t isz = i32 ? 4 : 8;
   const int k = (int)(c->host_calls & 1);
   const size_t noff = (size_t)c->T_r * (size_t)c->B + 1;
-  const int64_t nnz = h_offsets[noff - 1];
+  const int64_t nnz = i32 ? (int64_t) static_cast<const int32_t*>(h_offsets)[noff - 1]
+                          : static_cast<const int64_t*>(h_offsets)[noff - 1];
   if (nnz < 0) FAIL(c, EMB_ERR_ARG, "negative nnz");
-  if (!c->p_off[k] || (size_t)nnz > c->p_cap[k]) {  // (re)allocate stage k: drain everything first
+  if (!c->p_off[k] || noff * isz > c->p_offcap[k] || (size_t)nnz * isz > c->p_cap[k]) {
+    // (re)allocate stage k: drain everything first
     CK(c, cudaStreamSynchronize(c->s_in));
     CK(c, cudaStreamSynchronize(c->s_out));
     CK(c, cudaStreamSynchronize(s));
-    if (!c->p_off[k]) CK(c, cudaMalloc(&c->p_off[k], noff * sizeof(int64_t)));
+    if (c->p_off[k]) CK(c, cudaFree(c->p_off[k]));
     if (c->p_idx[k]) CK(c, cudaFree(c->p_idx[k]));
-    c->p_cap[k] = std::max<size_t>((size_t)nnz, 1) + (size_t)nnz / 4;
-    CK(c, cudaMalloc(&c->p_idx[k], c->p_cap[k] * sizeof(int64_t)));
+    c->p_offcap[k] = noff * 8;
+    c->p_cap[k] = (std::max<size_t>((size_t)nnz, 1) + (size_t)nnz / 4) * 8;
+    CK(c, cudaMalloc(&c->p_off[k], c->p_offcap[k]));
+    CK(c, cudaMalloc(&c->p_idx[k], c->p_cap[k]));
   }
   // 1. H2D into stage k once the kernel that last read it (two calls ago) is done
   if (c->kern_rec[k]) CK(c, cudaStreamWaitEvent(c->s_in, c->ev_kern[k], 0));
-  CK(c, cudaMemcpyAsync(c->p_off[k], h_offsets, noff * sizeof(int64_t), cudaMemcpyHostToDevice, c->s_in));
-  if (nnz > 0)
-    CK(c, cudaMemcpyAsync(c->p_idx[k], h_indices, (size_t)nnz * sizeof(int64_t), cudaMemcpyHostToDevice, c->s_in));
+  CK(c, cudaMemcpyAsync(c->p_off[k], h_offsets, noff * isz, cudaMemcpyHostToDevice, c->s_in));
+  if (nnz > 0) CK(c, cudaMemcpyAsync(c->p_idx[k], h_indices, (size_t)nnz * isz, cudaMemcpyHostToDevice, c->s_in));
   CK(c, cudaEventRecord(c->ev_in[k], c->s_in));
-  // 2. forward on the caller's stream after the inputs landed and after the D2H that last
-  //    read this epoch's output slot (2-slot ring) finished
-  const int slot = (int)((c->epoch + 1) & 1);
+  // 2. forward e on the caller's stream after its inputs landed and after the D2H of
+  //    Y_r(e-2) finished: a peer's forward e+1 may overwrite slot (e-2) % 3 as soon as
+  //    this rank's forward e has signalled (kOutSlots ring argument)
+  const uint64_t e = c->epoch + 1;
   CK(c, cudaStreamWaitEvent(s, c->ev_in[k], 0));
-  if (c->out_rec[slot]) CK(c, cudaStreamWaitEvent(s, c->ev_out[slot], 0));
+  if (e >= 3 && c->out_rec[(e - 2) % kOutSlots]) CK(c, cudaStreamWaitEvent(s, c->ev_out[(e - 2) % kOutSlots], 0));
   void* dout = nullptr;
-  emb_status_t st = emb_forward(c, c->p_off[k], c->p_idx[k], flags, stream, &dout);
+  emb_status_t st = forward_impl(c, c->p_off[k], c->p_idx[k], i32, flags & ~EMB_FWD_SEPARATE_WAIT, s, &dout);
   if (st != EMB_OK) return st;
-  if (flags & EMB_FWD_SEPARATE_WAIT) {
-    st = emb_wait(c, stream);
-    if (st != EMB_OK) return st;
-  }
   CK(c, cudaEventRecord(c->ev_kern[k], s));
   c->kern_rec[k] = true;
-  // 3. D2H of Y_r on the copy-out stream, overlapping the next call's H2D and kernel
+  // 3. D2H of Y_r(e) on the copy-out stream, overlapping the next call's H2D and kernel
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   CK(c, cudaStreamWaitEvent(c->s_out, c->ev_kern[k], 0));
+  if (c->d2h_delay_us > 0) emb_sleep_kernel<<<1, 1, 0, c->s_out>>>((uint64_t)c->d2h_delay_us * 1000ull);
   CK(c, cudaMemcpyAsync(h_out, dout, (size_t)Br * c->T * c->d * esize(c->odt), cudaMemcpyDeviceToHost, c->s_out));
-  CK(c, cudaEventRecord(c->ev_out[slot], c->s_out));
-  c->out_rec[slot] = true;
+  CK(c, cudaEventRecord(c->ev_out[e % kOutSlots], c->s_out));
+  c->out_rec[e % kOutSlots] = true;
   c->host_calls += 1;
   return EMB_OK;
+}
+
+emb_status_t emb_forward_host_async(emb_ctx_t* c, const int64_t* h_offsets, const int64_t* h_indices, uint32_t flags,
+                                    void* stream, void* h_out) {
+  return host_async_impl(c, h_offsets, h_indices, false, flags, (cudaStream_t)stream, h_out);
+}
+
+emb_status_t emb_forward_host_async_i32(emb_ctx_t* c, const int32_t* h_offsets, const int32_t* h_indices,
+                                        uint32_t flags, void* stream, void* h_out) {
+  return host_async_impl(c, h_offsets, h_indices, true, flags, (cudaStream_t)stream, h_out);
 }
 
 emb_status_t emb_host_drain(emb_ctx_t* c, void* stream) {
@@ -826,7 +829,7 @@ emb_status_t emb_host_drain(emb_ctx_t* c, void* stream) {
   if (!c->s_in) return EMB_OK;
   CK(c, cudaSetDevice(c->dev));
   cudaStream_t s = (cudaStream_t)stream;
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < kOutSlots; ++i)
     if (c->out_rec[i]) CK(c, cudaStreamWaitEvent(s, c->ev_out[i], 0));
   return EMB_OK;
 }
@@ -892,43 +895,50 @@ emb_status_t emb_backward_grad_ready(emb_ctx_t* c, void* stream) {
   return EMB_OK;
 }
 
-// f2, bwd_algo 1 (emb_bwd_sort.cuh): counting sort of the lookups by dW row, then a
-// segmented gather-sum with one red.add per run of equal rows
-static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int64_t* offsets, const int64_t* indices,
-                                    cudaStream_t s) {
+// f2, bwd_algo 1 (emb_bwd_sort.cuh): workspace of the radix sort, allocated before the
+// step is committed (a failure here must still release the peers, see emb_backward)
+static emb_status_t sorted_workspace(emb_ctx_t* c, const int64_t* offsets, cudaStream_t s) {
   if (!c->d_rowbase) {                                  // workspace sized by the local rows
     std::vector<int64_t> rb(c->T_r + 1, 0);
     for (int i = 0; i < c->T_r; ++i) rb[i + 1] = rb[i] + c->rows[c->local[i]];
-    if (rb[c->T_r] >= 0xffffffffll) FAIL(c, EMB_ERR_ARG, "bwd_algo 1: more than 2^32-2 local rows");
-    const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+    if (rb[c->T_r] >= (1ll << 27)) FAIL(c, EMB_ERR_ARG, "bwd_algo 1: more than 2^27 local rows (3 radix passes)");
     for (int g = 0; g < c->G; ++g)
       if ((c->bstart[g + 1] - c->bstart[g]) * (int64_t)c->T >= (1ll << 28))
-        FAIL(c, EMB_ERR_ARG, "bwd_algo 1: B_r * T must be < 2^28 (B_r = %lld)", (long long)Br);
+        FAIL(c, EMB_ERR_ARG, "bwd_algo 1: B_r * T must be < 2^28 (rank %d)", g);
     c->bs_R = rb[c->T_r];
-    c->bs_nblk = (c->bs_R + kScanTile - 1) / kScanTile;
     CK(c, cudaMalloc(&c->d_rowbase, rb.size() * sizeof(int64_t)));
     CK(c, cudaMemcpy(c->d_rowbase, rb.data(), rb.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
-    CK(c, cudaMalloc(&c->d_bcnt, std::max<int64_t>(c->bs_R, 1) * sizeof(uint32_t)));
-    CK(c, cudaMalloc(&c->d_bsum, std::max<int64_t>(c->bs_nblk, 1) * sizeof(uint32_t)));
   }
-  if (!c->d_pairs) {                                    // entry list: sized from the first CSR
+  if (!c->d_pairs) {                                    // entry lists: sized from the first CSR
     if (c->bs_cap <= 0) {                               // (one host sync, first call only)
       int64_t nnz = 0;
       CK(c, cudaMemcpyAsync(&nnz, offsets + (int64_t)c->T_r * c->B, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
       CK(c, cudaStreamSynchronize(s));
       c->bs_cap = std::min<int64_t>(nnz + nnz / 4 + 4096, 0xffffffffll);
     }
+    c->rs_nblk = (c->bs_cap + kRTile - 1) / kRTile;
+    const int64_t nh = (int64_t)kRBins * c->rs_nblk;
     CK(c, cudaMalloc(&c->d_pairs, (size_t)c->bs_cap * sizeof(uint2)));
+    CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_cap * sizeof(uint2)));
+    CK(c, cudaMalloc(&c->d_ghist, (size_t)nh * sizeof(uint32_t)));
+    CK(c, cudaMalloc(&c->d_rbsum, (size_t)((nh + kScanTile - 1) / kScanTile) * sizeof(uint32_t)));
   }
+  const size_t dsm = (size_t)(2 * kRTile + (2 + kBlock / 32) * kRBins) * sizeof(uint32_t);
+  CK(c, cudaFuncSetAttribute(emb_bradix_down_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm));
+  return EMB_OK;
+}
+
+// f2, bwd_algo 1: LSD radix sort of the lookups by dW row, then a segmented gather-sum
+// with one red.add per run of equal rows (workspace prepared by sorted_workspace)
+static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int64_t* offsets, const int64_t* indices,
+                                    cudaStream_t s) {
   SortParams q;
   memset(&q, 0, sizeof(q));
   q.offsets = offsets;
   q.indices = indices;
   q.rowbase = c->d_rowbase;
   q.tables = c->d_tables;
-  q.cnt = c->d_bcnt;
   q.pairs = c->d_pairs;
-  q.bsum = c->d_bsum;
   q.dW = bp.dW;
   for (int g = 0; g < kMaxG; ++g) {
     q.gsrc[g] = bp.gsrc[g];
@@ -947,65 +957,36 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   q.G = c->G;
   q.rank = c->rank;
   q.lanes = c->blanes;
-  q.chunk_rows = c->chunk_rows ? c->chunk_rows : 256;
+  q.chunk_rows = bp.chunk_rows;
   q.epoch = bp.epoch;
   const size_t tsm = (size_t)(c->T_r + 1) * 2 * sizeof(int64_t);
   const int grid = c->num_sms * 8;
-  if (c->bwd_algo == 3) {                               // LSD radix sort of the entries by row
-    if (!c->d_pairs_b) {
-      c->rs_nblk = (c->bs_cap + kRTile - 1) / kRTile;
-      const int64_t nh = (int64_t)kRBins * c->rs_nblk;
-      CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_cap * sizeof(uint2)));
-      CK(c, cudaMalloc(&c->d_ghist, (size_t)nh * sizeof(uint32_t)));
-      CK(c, cudaMalloc(&c->d_rbsum, (size_t)((nh + kScanTile - 1) / kScanTile) * sizeof(uint32_t)));
-    }
-    emb_bradix_gen_kernel<<<grid, kBlock, 0, s>>>(q);
-    int bits = 1;
-    while (bits < 32 && (1ll << bits) < c->bs_R) ++bits;
-    const int passes = (bits + kRBits - 1) / kRBits;
-    const int64_t nh = (int64_t)kRBins * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
-    const size_t dsm = (size_t)(2 * kRTile + (2 + kBlock / 32) * kRBins) * sizeof(uint32_t);
-    CK(c, cudaFuncSetAttribute(emb_bradix_down_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm));
-    uint2* in = c->d_pairs;
-    uint2* out = c->d_pairs_b;
-    q.ghist = c->d_ghist;
-    q.nblk_r = c->rs_nblk;
-    SortParams qs = q;                                  // the scan runs over the histograms
-    qs.cnt = c->d_ghist;
-    qs.R = nh;
-    qs.bsum = c->d_rbsum;
-    for (int ps = 0; ps < passes; ++ps) {
-      q.rin = in;
-      q.rout = out;
-      q.shift = kRBits * ps;
-      emb_bradix_up_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
-      emb_bsort_scan_sum_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
-      emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_rbsum, nb2);
-      emb_bsort_scan_apply_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
-      emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, dsm, s>>>(q);
-      std::swap(in, out);
-    }
-    q.pairs = in;                                       // sorted by row
-  } else {
-  CK(c, cudaMemsetAsync(c->d_bcnt, 0, (size_t)c->bs_R * sizeof(uint32_t), s));
-  const bool agg = c->bwd_algo == 2;                   // CTA-level shared-memory aggregation
-  const size_t hsm = (size_t)2 * kHashSlots * sizeof(uint32_t) + tsm;
-  const size_t ssm = (size_t)3 * kHashSlots * sizeof(uint32_t) + 1025 * sizeof(int64_t);
-  if (agg) {
-    CK(c, cudaFuncSetAttribute(emb_bsort_hist2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm));
-    CK(c, cudaFuncSetAttribute(emb_bsort_scatter2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm));
-    emb_bsort_hist2_kernel<<<c->num_sms * 3, kBlock, hsm, s>>>(q);
-  } else {
-    emb_bsort_hist_kernel<<<grid, kBlock, tsm, s>>>(q);
+  emb_bradix_gen_kernel<<<grid, kBlock, 0, s>>>(q);
+  int bits = 1;
+  while (bits < 32 && (1ll << bits) < c->bs_R) ++bits;
+  const int passes = (bits + kRBits - 1) / kRBits;
+  const int64_t nh = (int64_t)kRBins * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
+  const size_t dsm = (size_t)(2 * kRTile + (2 + kBlock / 32) * kRBins) * sizeof(uint32_t);
+  uint2* in = c->d_pairs;
+  uint2* out = c->d_pairs_b;
+  q.ghist = c->d_ghist;
+  q.nblk_r = c->rs_nblk;
+  SortParams qs = q;                                    // the scan runs over the histograms
+  qs.cnt = c->d_ghist;
+  qs.R = nh;
+  qs.bsum = c->d_rbsum;
+  for (int ps = 0; ps < passes; ++ps) {
+    q.rin = in;
+    q.rout = out;
+    q.shift = kRBits * ps;
+    emb_bradix_up_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
+    emb_bsort_scan_sum_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
+    emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_rbsum, nb2);
+    emb_bsort_scan_apply_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
+    emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, dsm, s>>>(q);
+    std::swap(in, out);
   }
-  if (c->bs_nblk > 0) {
-    emb_bsort_scan_sum_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
-    emb_bsort_scan_top_kernel<<<1, kBlock, 0, s>>>(c->d_bsum, c->bs_nblk);
-    emb_bsort_scan_apply_kernel<<<(unsigned)c->bs_nblk, kBlock, 0, s>>>(q);
-  }
-  if (agg) emb_bsort_scatter2_kernel<<<c->num_sms * 2, kBlock, ssm, s>>>(q);
-  else emb_bsort_scatter_kernel<<<grid, kBlock, 0, s>>>(q);
-  }
+  q.pairs = in;                                         // sorted by row
   void (*k)(SortParams) = nullptr;
   if (c->bvb == 8) k = emb_bsort_reduce_kernel<8, 1>;
   else if (c->bnv == 2) k = emb_bsort_reduce_kernel<16, 2>;
@@ -1018,47 +999,78 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   return EMB_OK;
 }
 
+// the kernel launches of emb_backward's chosen path (gpu_launches accounting)
+static int backward_launches(const emb_ctx_t* c) {
+  if (c->bwd_algo != 1 || c->T_r == 0) return 1;
+  int64_t R = 0;
+  for (int i = 0; i < c->T_r; ++i) R += c->rows[c->local[i]];
+  int bits = 1;
+  while (bits < 32 && (1ll << bits) < R) ++bits;
+  return 2 + 5 * ((bits + kRBits - 1) / kRBits);      // gen + passes x (up, 3 scan, down) + reduce
+}
+
 emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, void* const* dW,
                           uint32_t flags, void* stream) {
-  (void)flags;
   if (!c) return EMB_ERR_ARG;
   if (!c->registered || !c->bwd_enabled) FAIL(c, EMB_ERR_STATE, "backward not enabled (set enable_backward before registering)");
   if (!c->bwd_ready_pending) FAIL(c, EMB_ERR_STATE, "emb_backward without emb_backward_grad_ready");
-  if (c->T_r > 0 && (!offsets || !indices || !dW)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
+  if (flags != 0) FAIL(c, EMB_ERR_ARG, "emb_backward takes no flags (got 0x%x)", flags);
   CK(c, cudaSetDevice(c->dev));
   cudaStream_t s = (cudaStream_t)stream;
-  if (!c->d_dW) CK(c, cudaMalloc(&c->d_dW, std::max(c->T_r, 1) * sizeof(float*)));
+  BwdParams p;
+  fill_bwd_params(c, &p);
+  // Everything that can fail is checked and allocated BEFORE the step is committed; if it
+  // fails, the step still releases the "done" flags so the peers' next grad_slot does not
+  // time out, and the pending state is cleared so the next step can proceed.
+  auto abandon = [&](emb_status_t st) -> emb_status_t {
+    const std::string msg = c->err;
+    c->bwd_ready_pending = false;
+    if (c->G > 1) {
+      BwdParams r = p;
+      for (int g = 0; g < kMaxG; ++g) r.peer_ready[g] = p.peer_done[g];   // release "done reading"
+      emb_bwd_signal_kernel<<<1, 32, 0, s>>>(r);
+      cudaGetLastError();
+    }
+    c->err = msg;
+    return st;
+  };
+  if (c->T_r > 0 && (!offsets || !indices || !dW)) {
+    c->err = "NULL buffer";
+    return abandon(EMB_ERR_ARG);
+  }
+  if (!c->d_dW) {
+    cudaError_t e = cudaMalloc(&c->d_dW, std::max(c->T_r, 1) * sizeof(float*));
+    if (e != cudaSuccess) { c->err = cudaGetErrorString(e); return abandon(EMB_ERR_CUDA); }
+  }
   bool same = (int)c->h_dW.size() == c->T_r;
   for (int i = 0; same && i < c->T_r; ++i) same = c->h_dW[i] == dW[i];
   if (!same) {
     for (int i = 0; i < c->T_r; ++i)
-      if (!dW[i] || ((uintptr_t)dW[i]) % 16) FAIL(c, EMB_ERR_ARG, "dW[%d] NULL or not 16-byte aligned", i);
+      if (!dW[i] || ((uintptr_t)dW[i]) % 16) {
+        c->err = "dW[" + std::to_string(i) + "] NULL or not 16-byte aligned";
+        return abandon(EMB_ERR_ARG);
+      }
     c->h_dW.assign(dW, dW + c->T_r);
-    CK(c, cudaStreamSynchronize(s));
-    CK(c, cudaMemcpy(c->d_dW, c->h_dW.data(), c->T_r * sizeof(float*), cudaMemcpyHostToDevice));
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) e = cudaMemcpy(c->d_dW, c->h_dW.data(), c->T_r * sizeof(float*), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) { c->err = cudaGetErrorString(e); return abandon(EMB_ERR_CUDA); }
+  }
+  p.dW = c->d_dW;
+  const bool sorted = c->bwd_algo == 1 && c->T_r > 0;
+  if (sorted) {
+    emb_status_t st = sorted_workspace(c, offsets, s);
+    if (st != EMB_OK) return abandon(st);
   }
   c->bwd_ready_pending = false;
-  BwdParams p;
-  fill_bwd_params(c, &p);
-  if (c->bwd_algo >= 1 && c->T_r > 0 && c->T_r <= 2048)
-    return backward_sorted(c, p, offsets, indices, s);
+  if (sorted) return backward_sorted(c, p, offsets, indices, s);
   p.offsets = offsets;
   p.indices = indices;
   void (*k)(BwdParams) = nullptr;
   size_t smem = 0;
-  const bool cache_ok = c->bnv == 1;                  // cache variants: 256-B and 512-B rows
-  if (c->bwd_v2 && c->bwd_cache && cache_ok) {
-    const bool w16 = c->bvb == 16;
-    if (c->bwd_cache == 8) k = w16 ? emb_bwd_kernel<16, 1, true, 8> : emb_bwd_kernel<8, 1, true, 8>;
-    else if (c->bwd_cache == 16) k = w16 ? emb_bwd_kernel<16, 1, true, 16> : emb_bwd_kernel<8, 1, true, 16>;
-    else k = w16 ? emb_bwd_kernel<16, 1, true, 32> : emb_bwd_kernel<8, 1, true, 32>;
-    smem = (size_t)(kBlock / 32) * c->bwd_cache * (32 * c->bvb + 4);
+  if (c->bwd_cache && c->bnv == 1) {                     // cache variants: 256-B and 512-B rows
+    k = c->bvb == 16 ? emb_bwd_kernel<16, 1, 16> : emb_bwd_kernel<8, 1, 16>;
+    smem = (size_t)(kBlock / 32) * 16 * (32 * c->bvb + 4);
     CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  } else if (c->bwd_v2) {
-    if (c->bvb == 8) k = emb_bwd_kernel<8, 1, true>;
-    else if (c->bnv == 2) k = emb_bwd_kernel<16, 2, true>;
-    else if (c->bnv == 4) k = emb_bwd_kernel<16, 4, true>;
-    else k = emb_bwd_kernel<16, 1, true>;
   } else if (c->bvb == 8) k = emb_bwd_kernel<8, 1>;
   else if (c->bnv == 2) k = emb_bwd_kernel<16, 2>;
   else if (c->bnv == 4) k = emb_bwd_kernel<16, 4>;
@@ -1111,14 +1123,13 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
     if (c->p_idx[i]) cudaFree(c->p_idx[i]);
     if (c->ev_in[i]) cudaEventDestroy(c->ev_in[i]);
     if (c->ev_kern[i]) cudaEventDestroy(c->ev_kern[i]);
-    if (c->ev_out[i]) cudaEventDestroy(c->ev_out[i]);
   }
+  for (int i = 0; i < kOutSlots; ++i)
+    if (c->ev_out[i]) cudaEventDestroy(c->ev_out[i]);
   if (c->s_in) cudaStreamDestroy(c->s_in);
   if (c->trace) cudaFree(c->trace);
   if (c->d_dW) cudaFree(c->d_dW);
   if (c->d_rowbase) cudaFree(c->d_rowbase);
-  if (c->d_bcnt) cudaFree(c->d_bcnt);
-  if (c->d_bsum) cudaFree(c->d_bsum);
   if (c->d_pairs) cudaFree(c->d_pairs);
   if (c->d_pairs_b) cudaFree(c->d_pairs_b);
   if (c->d_ghist) cudaFree(c->d_ghist);
@@ -1158,11 +1169,8 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   i->epoch = c->epoch;
   int per_sm = c->ctas_per_sm;
   if (per_sm <= 0 && c->registered) {
-    const bool sx = sidx_on(c, false, false, false);
-    const bool ds = ds_on(c, false, false, false);
-    KernelFn k = ds ? pick_ds(c->wdt, c->odt, c->ds)
-                    : pick_kernel(c->wdt, c->odt, c->vb, c->nv, eff_unroll(c), false, eff_minblocks(c), full_row(c), sx);
-    const size_t smem = ds ? (size_t)(kBlock / 32) * 1024 : dyn_smem(c, sx);
+    KernelFn k = pick_kernel(c, fwd_mode(false, c->has_shard, c->tma_store != 0));
+    const size_t smem = fwd_smem(c, fwd_mode(false, c->has_shard, c->tma_store != 0));
     if (smem > 0) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, smem);
   }
@@ -1171,6 +1179,10 @@ emb_status_t emb_get_info(const emb_ctx_t* c, emb_info_t* i) {
   i->lanes = c->lanes;
   i->vec_bytes = c->vb;
   i->vecs_per_lane = c->nv;
+  i->out_slots = kOutSlots;
+  // kernels one call launches: the fused forward (+ the f3 combine); emb_backward's path
+  i->fwd_launches = 1 + (c->has_shard ? 1 : 0);
+  i->bwd_launches = c->registered && c->bwd_enabled ? backward_launches(c) : 0;
   return EMB_OK;
 }
 
@@ -1180,24 +1192,8 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
   else if (!strcmp(key, "ctas_per_sm")) { if (v < 0 || v > 32) FAIL(c, EMB_ERR_ARG, "ctas_per_sm"); c->ctas_per_sm = (int)v; }
   else if (!strcmp(key, "stagger")) c->stagger = v ? 1 : 0;
   else if (!strcmp(key, "timeout_ms")) { if (v < 1) FAIL(c, EMB_ERR_ARG, "timeout_ms < 1"); c->timeout_ns = v * 1000000ll; }
-  else if (!strcmp(key, "unroll")) {
-    if (v != 0 && v != 2 && v != 3 && v != 4 && v != 8 && v != 16 && v != -4 && v != -8 && v != -12 && v != -16)
-      FAIL(c, EMB_ERR_ARG, "unroll must be 2, 4 (register pipeline), 3 (2 x 8 rows, 16 warps/SM), 8, 16 (cp.async ring) "
-                           "or -4/-8/-12/-16 (ring v2)");
-    c->unroll = (int)v;
-  }
-  else if (!strcmp(key, "minblocks")) {
-    if (v != 0 && v != 1 && v != 4 && v != 5 && v != 6) FAIL(c, EMB_ERR_ARG, "minblocks must be 0 (auto), 1, 4, 5 or 6");
-    c->minblocks = (int)v;
-  }
-  else if (!strcmp(key, "sidx")) c->sidx = v ? 1 : 0;
-  else if (!strcmp(key, "ds")) {
-    if (v != 0 && v != 1 && v != 3 && v != 4) FAIL(c, EMB_ERR_ARG, "ds must be 0 (off, default), 1 or 4 (4 CTAs/SM), 3 (3 CTAs/SM)");
-    c->ds = (int)v;
-  }
   else if (!strcmp(key, "bwd_interleave")) c->bwd_interleave = v ? 1 : 0;
-  else if (!strcmp(key, "bwd_v2")) c->bwd_v2 = v ? 1 : 0;
-  else if (!strcmp(key, "bwd_algo")) { if (v < 0 || v > 3) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0, 1, 2 or 3"); c->bwd_algo = (int)v; }
+  else if (!strcmp(key, "bwd_algo")) { if (v < 0 || v > 1) FAIL(c, EMB_ERR_ARG, "bwd_algo must be 0 or 1"); c->bwd_algo = (int)v; }
   else if (!strcmp(key, "bwd_max_nnz")) {
     if (v < 0 || v >= (1ll << 32)) FAIL(c, EMB_ERR_ARG, "bwd_max_nnz not in [0, 2^32)");
     if (c->d_pairs) { cudaFree(c->d_pairs); c->d_pairs = nullptr; }
@@ -1207,16 +1203,18 @@ emb_status_t emb_set_option(emb_ctx_t* c, const char* key, int64_t v) {
     c->bs_cap = v;
   }
   else if (!strcmp(key, "bwd_cache")) {
-    if (v != 0 && v != 8 && v != 16 && v != 32) FAIL(c, EMB_ERR_ARG, "bwd_cache must be 0, 8, 16 or 32");
+    if (v != 0 && v != 16) FAIL(c, EMB_ERR_ARG, "bwd_cache must be 0 or 16");
     c->bwd_cache = (int)v;
   }
   else if (!strcmp(key, "bwd_chunk_rows")) { if (v < 0 || v > 65536) FAIL(c, EMB_ERR_ARG, "bwd_chunk_rows not in [0, 65536]"); c->bwd_chunk_rows = (int)v; }
   else if (!strcmp(key, "bwd_group")) { if (v < 0 || v > 4096) FAIL(c, EMB_ERR_ARG, "bwd_group not in [0, 4096]"); c->bwd_group = (int)v; }
   else if (!strcmp(key, "fwd_interleave")) c->fwd_interleave = v ? 1 : 0;
   else if (!strcmp(key, "tail_div")) { if (v < 1 || v > 64) FAIL(c, EMB_ERR_ARG, "tail_div not in [1, 64]"); c->tail_div = (int)v; }
-  else if (!strcmp(key, "row_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "row_l2 not in [0, 5]"); c->row_l2 = (int)v; }
-  else if (!strcmp(key, "out_l2")) { if (v < 0 || v > 5) FAIL(c, EMB_ERR_ARG, "out_l2 not in [0, 5]"); c->out_l2 = (int)v; }
   else if (!strcmp(key, "tma_store")) c->tma_store = v ? 1 : 0;
+  else if (!strcmp(key, "debug_d2h_delay_us")) {
+    if (v < 0 || v > 10000000) FAIL(c, EMB_ERR_ARG, "debug_d2h_delay_us not in [0, 1e7]");
+    c->d2h_delay_us = v;
+  }
   else if (!strcmp(key, "carveout")) {
     if (v < -1 || v > 100) FAIL(c, EMB_ERR_ARG, "carveout in [-1 (driver default), 100] percent");
     c->carveout = (int)v;
@@ -1264,16 +1262,27 @@ emb_status_t emb_baseline_splits(const emb_ctx_t* c, int64_t* send_counts, int64
   return EMB_OK;
 }
 
-emb_status_t emb_baseline_pool(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags,
-                               void* stream, void* send) {
+static emb_status_t baseline_pool_impl(emb_ctx_t* c, const void* offsets, const void* indices, bool i32, uint32_t flags,
+                                       cudaStream_t s, void* send) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_pool before emb_register_tables");
   if (c->has_shard) FAIL(c, EMB_ERR_ARG, "the comparison path does not support row-sharded tables");
   if (c->T_r > 0 && (!offsets || !indices || !send)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
   CK(c, cudaSetDevice(c->dev));
   FwdParams p;
-  fill_params(c, offsets, indices, false, (char*)send, &p);
-  return launch_fwd(c, p, flags & EMB_FWD_CHECK_BOUNDS, (cudaStream_t)stream);
+  fill_params(c, offsets, indices, i32, false, (char*)send, &p);
+  p.check = (flags & EMB_FWD_CHECK_BOUNDS) ? 1 : 0;
+  return launch_fwd(c, p, flags & EMB_FWD_CHECK_BOUNDS, s);
+}
+
+emb_status_t emb_baseline_pool(emb_ctx_t* c, const int64_t* offsets, const int64_t* indices, uint32_t flags,
+                               void* stream, void* send) {
+  return baseline_pool_impl(c, offsets, indices, false, flags, (cudaStream_t)stream, send);
+}
+
+emb_status_t emb_baseline_pool_i32(emb_ctx_t* c, const int32_t* offsets, const int32_t* indices, uint32_t flags,
+                                   void* stream, void* send) {
+  return baseline_pool_impl(c, offsets, indices, true, flags, (cudaStream_t)stream, send);
 }
 
 emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, void* out) {

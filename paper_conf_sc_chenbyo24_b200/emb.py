@@ -11,8 +11,8 @@ import ctypes as C
 from typing import Callable, List, Optional, Sequence, Tuple
 
 from . import _lib
-from ._lib import (EMB_BF16, EMB_DEVERR_BOUNDS, EMB_DEVERR_TIMEOUT, EMB_F32, EMB_FWD_CHECK_BOUNDS,  # noqa: F401
-                   EMB_FWD_SEPARATE_WAIT, STATUS_NAMES, EmbInfo)
+from ._lib import (EMB_BF16, EMB_DEVERR_BOUNDS, EMB_DEVERR_CAPACITY, EMB_DEVERR_TIMEOUT, EMB_F32,  # noqa: F401
+                   EMB_FWD_CHECK_BOUNDS, EMB_FWD_SEPARATE_WAIT, STATUS_NAMES, EmbInfo)
 
 
 class EmbError(RuntimeError):
@@ -56,6 +56,24 @@ def _stream(s) -> Optional[int]:
     if isinstance(s, int):
         return s
     return s.cuda_stream
+
+
+def _is_i32(offsets, indices) -> bool:
+    """Index width of a CSR given as torch tensors (int32 -> the *_i32 entry points, C12);
+    plain integer addresses are int64."""
+    wo = getattr(offsets, "dtype", None)
+    wi = getattr(indices, "dtype", None)
+    names = {str(wo), str(wi)} - {"None"}
+    if not names:
+        return False
+    if len(names) != 1:
+        raise TypeError(f"offsets and indices must have the same dtype, got {wo} and {wi}")
+    n = names.pop()
+    if n in ("torch.int32", "int32"):
+        return True
+    if n in ("torch.int64", "int64"):
+        return False
+    raise TypeError(f"offsets / indices must be int64 or int32, got {n}")
 
 
 def _check(ctx: Optional[EmbCtx], st: int) -> None:
@@ -128,9 +146,11 @@ def emb_register_sharded_tables(ctx: EmbCtx, rows: Sequence[int], num_shards: Se
 
 
 def emb_forward(ctx: EmbCtx, offsets, indices, flags: int = 0, stream=None) -> int:
-    """Returns the device address of this epoch's Y_r = [B_r][T][d]."""
+    """Returns the device address of this epoch's Y_r = [B_r][T][d] (int32 tensors call
+    emb_forward_i32)."""
     out = C.c_void_p()
-    st = _lib.lib().emb_forward(ctx, _ptr(offsets), _ptr(indices), int(flags), _stream(stream), C.byref(out))
+    fn = _lib.lib().emb_forward_i32 if _is_i32(offsets, indices) else _lib.lib().emb_forward
+    st = fn(ctx, _ptr(offsets), _ptr(indices), int(flags), _stream(stream), C.byref(out))
     _check(ctx, st)
     return out.value
 
@@ -146,9 +166,10 @@ def emb_forward_host(ctx: EmbCtx, h_offsets, h_indices, h_out, flags: int = 0, s
 
 
 def emb_forward_host_async(ctx: EmbCtx, h_offsets, h_indices, h_out, flags: int = 0, stream=None) -> None:
-    """Pipelined host path: H2D / kernel / D2H of consecutive calls overlap."""
-    st = _lib.lib().emb_forward_host_async(ctx, _ptr(h_offsets), _ptr(h_indices), int(flags), _stream(stream),
-                                           _ptr(h_out))
+    """Pipelined host path: H2D / kernel / D2H of consecutive calls overlap (int32 host
+    tensors call emb_forward_host_async_i32)."""
+    fn = _lib.lib().emb_forward_host_async_i32 if _is_i32(h_offsets, h_indices) else _lib.lib().emb_forward_host_async
+    st = fn(ctx, _ptr(h_offsets), _ptr(h_indices), int(flags), _stream(stream), _ptr(h_out))
     _check(ctx, st)
 
 
@@ -224,7 +245,8 @@ def emb_baseline_splits(ctx: EmbCtx) -> Tuple[List[int], List[int]]:
 
 
 def emb_baseline_pool(ctx: EmbCtx, offsets, indices, send, flags: int = 0, stream=None) -> None:
-    _check(ctx, _lib.lib().emb_baseline_pool(ctx, _ptr(offsets), _ptr(indices), int(flags), _stream(stream), _ptr(send)))
+    fn = _lib.lib().emb_baseline_pool_i32 if _is_i32(offsets, indices) else _lib.lib().emb_baseline_pool
+    _check(ctx, fn(ctx, _ptr(offsets), _ptr(indices), int(flags), _stream(stream), _ptr(send)))
 
 
 def emb_baseline_unpack(ctx: EmbCtx, recv, out, stream=None) -> None:

@@ -13,7 +13,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def _declared(header):
     src = open(os.path.join(ROOT, "include", header)).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b((?:emb|synth)_[a-z_]+)\s*\(", src)) - {"emb_allgather_fn"})
+    return sorted(set(re.findall(r"\b((?:emb|synth)_[a-z0-9_]+)\s*\(", src)) - {"emb_allgather_fn"})
 
 
 def _exported(so):

@@ -104,11 +104,11 @@ def test_bwd_placement_invariance():
 
 
 @pytest.mark.parametrize("opts", [{"bwd_interleave": 0}, {"bwd_group": 2}, {"bwd_group": 3}, {"bwd_group": 4},
-                                  {"bwd_group": 7}, {"bwd_group": 1}, {"bwd_v2": 1}, {"bwd_v2": 1, "bwd_group": 3},
-                                  {"bwd_v2": 1, "bwd_interleave": 0}, {"bwd_v2": 1, "bwd_cache": 8},
-                                  {"bwd_v2": 1, "bwd_cache": 16, "bwd_chunk_rows": 1024},
-                                  {"bwd_v2": 1, "bwd_cache": 32, "bwd_interleave": 0}, {"bwd_algo": 1},
-                                  {"bwd_algo": 2}, {"bwd_algo": 3}])
+                                  {"bwd_group": 7}, {"bwd_group": 1}, {"bwd_cache": 0}, {"bwd_cache": 0, "bwd_group": 3},
+                                  {"bwd_cache": 0, "bwd_interleave": 0},
+                                  {"bwd_cache": 16, "bwd_chunk_rows": 1024},
+                                  {"bwd_cache": 16, "bwd_interleave": 0}, {"bwd_algo": 1},
+                                  {"bwd_algo": 1, "bwd_chunk_rows": 7}])
 def test_bwd_chunk_orders_integer_exact(opts):
     """every chunk order (table-major, groups of g tables incl. a ragged last group, all
     tables interleaved) visits every bag exactly once: exact on integer gradients"""
@@ -120,12 +120,13 @@ def test_bwd_chunk_orders_integer_exact(opts):
         assert np.array_equal(got[t].astype(np.float64), ref[t]), t
 
 
-@pytest.mark.parametrize("dim,cache", [(16, 8), (64, 16), (128, 32), (256, 8), (16, -1), (64, -1), (128, -1),
-                                       (256, -1), (512, -1), (64, -3), (128, -3)])
+@pytest.mark.parametrize("dim,cache", [(16, 16), (64, 16), (128, 16), (256, 16), (16, 0), (128, 0), (512, 0),
+                                       (16, -1), (64, -1), (128, -1), (256, -1), (512, -1)])
 def test_bwd_row_cache_exact_and_float_bound(dim, cache):
-    """f2 per-warp dW row cache (bwd_cache): integer gradients exact, float gradients within
-    the order-independent summation bound (cached rows are summed in shared memory first)"""
-    opts = {"bwd_v2": 1, "bwd_cache": cache, "bwd_chunk_rows": 512} if cache > 0 else {"bwd_algo": -cache}
+    """f2 per-warp dW row cache (bwd_cache) and the sorted algorithm (cache -1 = bwd_algo 1):
+    integer gradients exact, float gradients within the order-independent summation bound
+    (cached rows are summed in shared memory first)"""
+    opts = {"bwd_cache": cache, "bwd_chunk_rows": 512} if cache >= 0 else {"bwd_algo": -cache}
     w = synth.make_workload("tiny", G=2, pmin=0, pmax=60, B=150, T=3, dim=dim, rows=200, dist="zipf")
     got, offs, idxs = _run_bwd(w, _dY(w, 21, integer=True), 22, opts=opts)
     ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, _dY(w, 21, integer=True), w.B, w.G)
@@ -140,12 +141,10 @@ def test_bwd_row_cache_exact_and_float_bound(dim, cache):
         assert np.all(err <= n * 2.0 ** -24 * 2 * S[t] + 1e-30), t
 
 
-@pytest.mark.parametrize("G,dist,algo", [(1, "zipf", 1), (2, "uniform", 1), (3, "zipf", 1), (1, "zipf", 2),
-                                          (2, "uniform", 2), (3, "zipf", 2), (1, "zipf", 3), (2, "uniform", 3),
-                                          (3, "zipf", 3)])
+@pytest.mark.parametrize("G,dist,algo", [(1, "zipf", 1), (2, "uniform", 1), (3, "zipf", 1)])
 def test_bwd_sorted_algo_integer_exact_multi_epoch(G, dist, algo):
-    """bwd_algo 1 (counting sort + segmented sum): exact on integer gradients over 3 epochs
-    (workspace reuse, counters re-zeroed), incl. empty bags and G > 1 one-sided dY loads"""
+    """bwd_algo 1 (radix sort + segmented sum): exact on integer gradients over 3 epochs
+    (workspace reuse), incl. empty bags and G > 1 one-sided dY loads"""
     w = synth.make_workload("tiny", G=G, pmin=0, pmax=70, B=131, T=5, dim=128, rows=400, dist=dist)
     dY = _dY(w, 31, integer=True)
     got, offs, idxs = _run_bwd(w, dY, 32, epochs=3, opts={"bwd_algo": algo})

@@ -48,9 +48,10 @@ def _layers(w, tabs_np, options=None):
                                                   w.odtype, grp.allgather_for(r), options))
 
 
-def _run(w, layers, csr_np, flags=0, streams=None):
+def _run(w, layers, csr_np, flags=0, streams=None, i32=False):
     offs, idxs = csr_np
-    dev_in = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(w.G)]
+    dt = torch.int32 if i32 else torch.int64
+    dev_in = [(torch.from_numpy(offs[r]).to(DEV).to(dt), torch.from_numpy(idxs[r]).to(DEV).to(dt)) for r in range(w.G)]
     streams = streams or [torch.cuda.Stream() for _ in range(w.G)]
     torch.cuda.synchronize()
     ys = []
@@ -202,16 +203,20 @@ def test_epoch_ring_poisoned_slots_exactly_once():
         _close(layers)
 
 
-def test_bounds_check_flag():
+@pytest.mark.parametrize("i32", [False, True])
+def test_bounds_check_flag(i32):
+    """EMB_FWD_CHECK_BOUNDS: out-of-range ids (past the end, negative) are skipped and flagged;
+    the result equals the oracle's pooling of the remaining ids, compared bit for bit."""
     w = synth.make_workload("tiny", G=1, pmin=1, pmax=6, B=40, T=2, dim=16, rows=100)
     tabs = H.np_tables(w)
     offs, idxs = H.np_csrs(w, 8)
     bad = idxs[0].copy()
     bad[3] = 100          # out of range
     bad[7] = -5
+    bad[8] = 2 ** 31 - 1 if i32 else 2 ** 40
     layers = _layers(w, tabs)
     try:
-        got = _run(w, layers, ([offs[0]], [bad]), E.EMB_FWD_CHECK_BOUNDS)[0]
+        got = _run(w, layers, ([offs[0]], [bad]), E.EMB_FWD_CHECK_BOUNDS, i32=i32)[0]
         assert layers[0].device_error(clear=True) & E.EMB_DEVERR_BOUNDS
         assert layers[0].device_error() == 0
     finally:
@@ -222,7 +227,7 @@ def test_bounds_check_flag():
         for b in range(w.B):
             js = [j for j in range(lo + o[b], lo + o[b + 1]) if 0 <= bad[j] < 100]
             exp = O.pool_bag_f32(tabs[t][bad[js]]) if js else np.zeros(w.dim, np.float32)
-            assert np.array_equal(np.abs(got[b, t]), np.abs(exp))
+            assert np.array_equal(got[b, t].view(np.uint32), exp.view(np.uint32)), (t, b)
 
 
 def test_peer_timeout_sets_error_instead_of_hanging():
@@ -327,32 +332,34 @@ def test_api_errors():
         E.emb_finalize(ctx)
 
 
-VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),
-                 dict(dim=64, pmin=1, pmax=40, B=257, rows=2000),
+VARIANT_CASES = [dict(dim=128, pmin=0, pmax=70, B=333, rows=3000, dist="zipf"),       # 512-B rows, 16-B lanes
+                 dict(dim=64, pmin=1, pmax=40, B=257, rows=2000),                     # 256-B rows, 8-B lanes
                  dict(dim=128, wdtype="bf16", odtype="bf16", pmin=0, pmax=50, B=129, rows=1000),
-                 dict(dim=32, pmin=0, pmax=9, B=100)]
+                 dict(dim=32, pmin=0, pmax=9, B=100),                                 # 128 B: 8 of 32 lanes
+                 dict(dim=6, pmin=0, pmax=12, B=77, rows=300),                        # 24 B: 8-B lanes, 3 active
+                 dict(dim=256, pmin=0, pmax=33, B=91, rows=700),                      # 1 KB: 2 vectors per lane
+                 dict(dim=512, wdtype="bf16", odtype="f32", pmin=0, pmax=20, B=65, rows=400)]   # 1 KB bf16
 
 
-@pytest.mark.parametrize("opts", [{"unroll": 2}, {"unroll": 4}, {"unroll": 8}, {"unroll": 16},
-                                  {"unroll": 4, "minblocks": 1}, {"unroll": 4, "minblocks": 6},
-                                  {"chunk_rows": 1}, {"chunk_rows": 100000}, {"stagger": 0}, {"sidx": 0},
-                                  {"sidx": 0, "unroll": 2}, {"sidx": 1, "chunk_rows": 7}, {"sidx": 0, "chunk_rows": 7},
-                                  {"ds": 1}, {"ds": 3}, {"ds": 1, "chunk_rows": 3}, {"ds": 1, "tail_div": 1}, {"fwd_interleave": 1},
-                                  {"tma_store": 1}, {"tma_store": 1, "chunk_rows": 3}, {"unroll": -8}, {"unroll": -16},
-                                  {"unroll": -12, "chunk_rows": 5}])
+@pytest.mark.parametrize("opts", [{}, {"chunk_rows": 1}, {"chunk_rows": 100000}, {"chunk_rows": 7}, {"chunk_rows": 3},
+                                  {"stagger": 0}, {"fwd_interleave": 1}, {"tail_div": 1}, {"tail_div": 16},
+                                  {"carveout": -1}, {"ctas_per_sm": 1}, {"tma_store": 1},
+                                  {"tma_store": 1, "chunk_rows": 3}])
+@pytest.mark.parametrize("i32", [False, True])
 @pytest.mark.parametrize("case", range(len(VARIANT_CASES)))
-def test_pipeline_variants_bitexact(opts, case):
-    """Every register/shared-memory pipeline variant and chunking is bit-exact."""
+def test_pipeline_variants_bitexact(opts, i32, case):
+    """Every row tiling x chunking x store variant x index width is bit-exact, with and
+    without the bounds-checking (per-id validity) kernel."""
     w = synth.make_workload("tiny", G=2, T=5, **VARIANT_CASES[case])
-    if (opts.get("tma_store") or opts.get("unroll", 0) < 0) and w.dim * w.elem_bytes() < 256:
-        pytest.skip("tma_store / ring v2 need full-warp rows (256 B+)")
+    if opts.get("tma_store") and w.dim * w.elem_bytes() not in (256, 512):
+        pytest.skip("tma_store needs rows of exactly one vector per lane (256 or 512 B)")
     tabs = H.np_tables(w)
     csr = H.np_csrs(w, 71)
     ref = H.oracle_outputs(w, 71, tabs, csr)
     layers = _layers(w, tabs, options=opts)
     try:
-        got = _run(w, layers, csr)
-        got_chk = _run(w, layers, csr, E.EMB_FWD_CHECK_BOUNDS)
+        got = _run(w, layers, csr, i32=i32)
+        got_chk = _run(w, layers, csr, E.EMB_FWD_CHECK_BOUNDS, i32=i32)
         for r in range(w.G):
             _assert_exact(got[r], ref[r])
             _assert_exact(got_chk[r], ref[r])

@@ -63,9 +63,8 @@ def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1, opts=None):
             s.synchronize()
             got = y.cpu().numpy()
             ok = ok and np.array_equal(got.view(np.uint32), ref.view(np.uint32))
-            y.fill_(float("nan"))
+            y.fill_(float("nan"))                     # poison: every epoch must rewrite its slot
             torch.cuda.synchronize()
-            dist.barrier()  # consumer of slot e&1 done before anyone runs e+2 (stream order across processes)
         err = layer.device_error()
         layer.close()
         dist.destroy_process_group()
@@ -78,7 +77,7 @@ def _worker(rank, G, port, q, flags, owner, epochs, delay_rank=-1, opts=None):
 @pytest.mark.parametrize("G,flags,owner,delay,opts", [(2, 0, None, -1, None), (3, 0, [2, 2, 0, 1, 0, 2], -1, None),
                                                      (2, 2, None, -1, None), (3, 0, None, 1, None), (2, 2, None, 0, None),
                                                      (3, 0, None, -1, {"tma_store": 1}),
-                                                     (2, 0, None, -1, {"unroll": -8})])
+                                                     (2, 0, None, -1, {"chunk_rows": 5, "tail_div": 1})])
 def test_cross_process_ipc_pgas(G, flags, owner, delay, opts):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
@@ -95,6 +94,73 @@ def test_cross_process_ipc_pgas(G, flags, owner, delay, opts):
     for rank, ok, err, tb in sorted(res):
         assert tb == "", tb
         assert ok, f"rank {rank} output != oracle"
+        assert err == 0, f"rank {rank} device error {err}"
+
+
+def _async_worker(rank, G, port, q, epochs, slow_rank, i32):
+    """emb_forward_host_async over real IPC, one rank's copy-out stream stalled before every
+    D2H: a peer racing ahead must not overwrite a slot that is still being copied out
+    (3-slot output ring)."""
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    try:
+        import torch.distributed as dist
+
+        import emb_test_helpers as H
+        import synth
+        from paper_conf_sc_chenbyo24_b200 import emb as E
+        from paper_conf_sc_chenbyo24_b200.comm import torch_allgather
+        from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
+
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=G)
+        w = synth.make_workload("tiny", G=G, pmin=0, pmax=25, B=96, T=6, dim=64, rows=600)
+        tabs = H.np_tables(w)
+        dev = torch.device("cuda", 0)
+        local = [torch.from_numpy(tabs[int(w.phys[t])]).to(dev) for t in w.local_tables(rank)]
+        opts = {"timeout_ms": 30000}
+        if rank == slow_rank:
+            opts["debug_d2h_delay_us"] = 40000
+        layer = PgasEmbedding(rank, G, 0, w.rows, w.owner, w.dim, local, w.B, "f32", "f32", torch_allgather(), opts)
+        dt = torch.int32 if i32 else torch.int64
+        hin, houts, refs = [], [], []
+        for ep in range(epochs):
+            o, x = synth.rank_csr(w, 700 + ep, rank)
+            hin.append((torch.from_numpy(o).to(dt).pin_memory(), torch.from_numpy(x).to(dt).pin_memory()))
+            houts.append(torch.full((layer.B_r, w.T, w.dim), float("nan")).pin_memory())
+            refs.append(H.oracle_outputs(w, 700 + ep, tabs)[rank])
+        s = torch.cuda.Stream()
+        for ep in range(epochs):
+            E.emb_forward_host_async(layer.ctx, hin[ep][0], hin[ep][1], houts[ep], 0, s)
+        E.emb_host_drain(layer.ctx, s)
+        s.synchronize()
+        ok = all(np.array_equal(houts[ep].numpy().view(np.uint32), refs[ep].view(np.uint32)) for ep in range(epochs))
+        err = layer.device_error()
+        dist.barrier()
+        layer.close()
+        dist.destroy_process_group()
+        q.put((rank, bool(ok), int(err), ""))
+    except Exception:
+        import traceback
+        q.put((rank, False, -1, traceback.format_exc()))
+
+
+@pytest.mark.parametrize("G,slow_rank,i32", [(2, 1, False), (3, 0, True)])
+def test_cross_process_host_async_slow_consumer(G, slow_rank, i32):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_async_worker, args=(r, G, port, q, 7, slow_rank, i32)) for r in range(G)]
+    for p in ps:
+        p.start()
+    res = sorted(q.get(timeout=300) for _ in range(G))
+    for p in ps:
+        p.join(timeout=60)
+    for rank, ok, err, tb in res:
+        assert tb == "", tb
+        assert ok, f"rank {rank} host output != oracle"
         assert err == 0, f"rank {rank} device error {err}"
 
 

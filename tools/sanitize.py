@@ -52,8 +52,8 @@ for G in (1, 2):
     for r in range(G):
         layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
     torch.cuda.synchronize()
-    # sorted backward algorithms (counting sort / radix sort + segmented sum), same slots and flags
-    for algo in (1, 3):
+    # sorted backward algorithm (radix sort + segmented sum), same slots and flags
+    for algo in (1,):
         for r in range(G):
             E.emb_set_option(layers[r].ctx, "bwd_algo", algo)
             with torch.cuda.stream(streams[r]):

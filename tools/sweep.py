@@ -44,7 +44,8 @@ def main():
         nnz = np.mean([int(b[0][-1]) for b in bs])
         byt = nnz * (w.dim * w.elem_bytes() + 8) + w.T * w.B * (8 + w.dim * w.out_elem_bytes())
         for o in [o for _ in range(a.repeat) for o in a.opts]:
-            defaults = {"chunk_rows": 0, "minblocks": 0, "unroll": 0, "ctas_per_sm": 0, "stagger": 1, "sidx": 1, "carveout": 0, "fwd_interleave": 0, "tma_store": 0, "tail_div": 4, "ds": 0}
+            defaults = {"chunk_rows": 0, "ctas_per_sm": 0, "stagger": 1, "carveout": 0, "fwd_interleave": 0,
+                        "tma_store": 0, "tail_div": 4}
             kv = dict(defaults)
             for item in o.split(",") if o else []:
                 k, v = item.split("=")
