@@ -2,16 +2,18 @@
 """Benchmark of the PGAS-style EMB-layer forward (BASELINE.json metric: EMB fwd
 samples/sec at 1/2/4/8 B200, max over ranks, + % of the HBM/NVLink roofline).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config weak|single|strong|weak_paper|tiny]
-                    [--dist zipf|uniform] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config weak|single|strong|weak_paper|large_shard|tiny]
+                    [--dist zipf|uniform] [--impl ours|reference] [--index-bits 64|32] [--shards S]
     torchrun --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
 
 One JSON line on rank 0.  A "step" is one whole EMB forward (lookup + pool + MP->DP
 exchange, PAPER.md L197 timed scope) over one batch of synthetic Criteo-shaped input
-already resident in HBM; `e2e` repeats it through emb_forward_host with pinned host
-CSR in and the host output out.  `--impl reference` times the CPU oracle (this tier's
-reference arm) on a bounded sample of the same workload.  Nothing here reads
-/root/reference.
+already resident in HBM.  Every timed figure is the median of `--repeats` (5) runs of K
+steps, each bracketed by a barrier + synchronize, device-timed with CUDA events on the
+launching stream and max-reduced over ranks (SURVEY §8(d) timing protocol); the clocks of
+every repeat are recorded.  `e2e` repeats it through the public C ABI with pinned host CSR
+in and the host output out.  `--impl reference` times the CPU oracle (this tier's reference
+arm) on a bounded sample of the same workload.  Nothing here reads /root/reference.
 """
 from __future__ import annotations
 
@@ -39,20 +41,24 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=100)
     p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--repeats", type=int, default=5, help="timed repeats of K steps; the median is reported")
     p.add_argument("--config", default="weak")
     p.add_argument("--dist", default=None, help="override index distribution (zipf|uniform)")
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--mode", default="forward", choices=["forward", "backward"],
                    help="backward = SURVEY row f2 (emb_backward: pull output gradients, scatter into dW)")
+    p.add_argument("--index-bits", type=int, default=64, choices=[64, 32],
+                   help="CSR index/offset width (C12: int64 is the paper's; int32 halves the index bytes)")
     p.add_argument("--batches", type=int, default=4, help="distinct pre-generated batches cycled")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-control", action="store_true", help="skip the uniform-index control measurement")
     p.add_argument("--no-compare", action="store_true", help="skip the NCCL comparison path")
+    p.add_argument("--no-trace", action="store_true", help="skip the f1 communication-timeline summary")
     p.add_argument("--opt", action="append", default=[], help="libemb option key=value")
     p.add_argument("--shards", type=int, default=1,
-                   help="f3: split every table into this many row shards (owners round-robin from the table's owner);"
-                        " the kernel partitions the full CSR in-kernel and combines partials in shard order")
+                   help="f3: split every table into this many row shards, shard s of table t on rank "
+                        "(owner[t] + s) %% N; the kernel partitions the full CSR in-kernel and combines partials")
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                    help="process-group backend (gloo: test harness only; a2a staged through host)")
     p.add_argument("--same-device", action="store_true",
@@ -68,42 +74,44 @@ def hbm_peak():
         return HBM_FALLBACK, "fallback"
 
 
-def config_desc(w, N):
+def config_desc(w, N, args):
     return {"workload": w.name, "tables_total": int(w.T), "tables_per_gpu": int(w.T // max(N, 1)) if w.name != "large" else None,
             "rows_per_table": int(w.rows[0]), "dim": w.dim, "global_batch": int(w.B), "local_batch": int(w.B // N),
             "pooling": f"U{{{w.pmin}..{w.pmax}}}", "indices": f"{w.dist}({w.alpha})" if w.dist == "zipf" else "uniform",
             "weights": w.wdtype, "out": w.odtype, "parallelism": f"table-wise MP x{N} + batch DP x{N}",
+            "index_bits": args.index_bits,
             "aliased": int(w.T // (int(w.phys.max()) + 1)) if int(w.phys.max()) + 1 < w.T else 1,
             "l2": "inputs larger than L2 (tables >> 126 MB, rotating CSR batches); no flush",
-            "row_shards_per_table": getattr(w, "_shards", 1)}
+            "row_shards_per_table": args.shards, "options": args.opt}
 
 
-def unique_rows(w, rank, batch):
+def unique_rows(w, tables_of_rank, batch, ranges=None):
     """Distinct (table, row) pairs a batch touches: the rows that must come from HBM
-    at least once (compulsory traffic under zipf reuse)."""
+    at least once (compulsory traffic under zipf reuse).  ranges[i] = (lo, hi): only ids of
+    that row range count (f3: a shard loads only its own rows)."""
     import torch
     off, idx = batch
-    lt = w.local_tables(rank)
     starts = off[:: w.B].tolist()
     tot = 0
-    for i in range(len(lt)):
+    for i in range(len(tables_of_rank)):
         seg = idx[starts[i]: starts[i + 1]]
+        if ranges is not None:
+            lo, hi = ranges[i]
+            seg = seg[(seg >= lo) & (seg < hi)]
         if seg.numel():
             tot += int(torch.unique(seg).numel())
     return tot
 
 
-def compulsory_bytes(w, uniq, nnz, nbags):
+def compulsory_bytes(w, uniq, nnz, nbags, ib):
     """Unique rows once + every index + every offset + every output vector written."""
-    return uniq * w.dim * w.elem_bytes() + nnz * 8 + nbags * (8 + w.dim * w.out_elem_bytes())
+    return uniq * w.dim * w.elem_bytes() + nnz * ib + nbags * (ib + w.dim * w.out_elem_bytes())
 
 
-def algorithmic_bytes(w, nnz, nbags, remote_bags):
-    """per lookup d*e + 8 (row + index); per bag 8 (offset) + d*e_o (output)."""
+def algorithmic_bytes(w, nnz, nbags, ib):
+    """per lookup d*e + index; per bag one offset + d*e_o (output)."""
     e, eo = w.elem_bytes(), w.out_elem_bytes()
-    hbm = nnz * (w.dim * e + 8) + nbags * (8 + w.dim * eo)
-    nvl = remote_bags * w.dim * eo
-    return hbm, nvl
+    return nnz * (w.dim * e + ib) + nbags * (ib + w.dim * eo)
 
 
 # ------------------------------------------------------------------------------ clocks
@@ -256,7 +264,7 @@ def reference_arm(args):
             "n_gpus": N, "steps": args.steps, "warmup": args.warmup, "ms_per_step": sec * 1e3,
             "higher_is_better": True, "scaling": "weak" if args.config.startswith("weak") else "strong",
             "vs_baseline": None, "dtype": "f32" if w.wdtype == "f32" else "bf16", "data": "synthetic",
-            "config": config_desc(w, N),
+            "config": config_desc(w, N, args),
             "cpu_baseline": {"value": val, "unit": "samples/s", "cores": cb["cores"], "kind": "oracle",
                              "sample": "per step: " + cb["sample"]},
             "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -265,13 +273,151 @@ def reference_arm(args):
     return 0
 
 
-# ------------------------------------------------------------------------------ backward (f2)
-def run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq, nbags, remote_bags, barrier, timed):
+# ------------------------------------------------------------------------------ f1 trace summary
+def trace_summary(tr, bins=40):
+    """f1 (Figs. 7/10): how the rank's stores spread over its kernel span.
+    tr: uint64 [n, 2] records {globaltimer ns, remote bytes << 32 | local bytes}."""
+    if tr.shape[0] == 0:
+        return {"records": 0}
+    t = tr[:, 0].astype(np.int64)
+    rem = (tr[:, 1] >> np.uint64(32)).astype(np.int64)
+    loc = (tr[:, 1] & np.uint64(0xFFFFFFFF)).astype(np.int64)
+    r0, r1 = int(t.min()), int(t.max())
+    e = np.linspace(r0, r1 + 1, bins + 1)
+    hr, _ = np.histogram(t, bins=e, weights=rem)
+    ha, _ = np.histogram(t, bins=e, weights=rem + loc)
+    cum = np.cumsum(hr) / max(hr.sum(), 1)
+    cuma = np.cumsum(ha) / max(ha.sum(), 1)
+    return {"records": int(tr.shape[0]), "span_us": (r1 - r0) / 1e3, "t0_ns": r0, "remote_bytes": int(rem.sum()),
+            "local_bytes": int(loc.sum()),
+            "remote_frac_by_quarter": [round(float(cum[int(bins * q) - 1]), 4) for q in (0.25, 0.5, 0.75, 1.0)],
+            "all_frac_by_quarter": [round(float(cuma[int(bins * q) - 1]), 4) for q in (0.25, 0.5, 0.75, 1.0)],
+            "remote_bins_nonzero_frac": float((hr > 0).mean()),
+            "remote_cv_over_bins": float(hr.std() / hr.mean()) if hr.mean() > 0 else None,
+            "remote_bytes_per_bin": hr.astype(int).tolist()}
+
+
+# ------------------------------------------------------------------------------ GPU arm
+class Harness:
+    """Process-group, stream and timing plumbing of one rank."""
+
+    def __init__(self, args):
+        import torch
+        import torch.distributed as dist
+        self.torch, self.dist, self.args = torch, dist, args
+        self.N = args.gpus
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        if world != self.N:
+            raise SystemExit(f"--gpus {self.N} but WORLD_SIZE={world}")
+        if args.same_device:
+            self.local = 0
+        torch.cuda.set_device(self.local)
+        self.dev = torch.device("cuda", self.local)
+        if self.N > 1:
+            if args.backend == "nccl":
+                dist.init_process_group("nccl", device_id=self.dev)
+            else:
+                dist.init_process_group("gloo")
+        self.stream = torch.cuda.Stream(device=self.dev)
+        self.clock_log = []
+
+    def barrier(self):
+        if self.N > 1:
+            self.dist.barrier()
+        self.torch.cuda.synchronize()
+
+    def allreduce_max(self, x):
+        if self.N == 1:
+            return float(x)
+        t = self.torch.tensor([float(x)], dtype=self.torch.float64,
+                              device=self.dev if self.args.backend == "nccl" else "cpu")
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def gather(self, obj):
+        if self.N == 1:
+            return [obj]
+        out = [None] * self.N
+        self.dist.all_gather_object(out, obj)
+        return out
+
+    def timed_once(self, fn, steps, finish=None):
+        torch = self.torch
+        self.barrier()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(self.stream)
+        for s in range(steps):
+            fn(s)
+        if finish is not None:
+            finish()
+        ev1.record(self.stream)
+        torch.cuda.synchronize()
+        return self.allreduce_max(ev0.elapsed_time(ev1) / steps)
+
+    def timed(self, fn, steps, finish=None, what="main"):
+        """median over `repeats` device-timed runs of `steps` steps (max over ranks each)"""
+        reps = []
+        for _ in range(max(self.args.repeats, 1)):
+            with ClockSampler(self.local) as clk:
+                ms = self.timed_once(fn, steps, finish)
+            reps.append({"ms": ms, **{k: v for k, v in clk.summary().items() if k in ("sm_mhz", "reasons")}})
+        self.clock_log.append({"what": what, "repeats": reps})
+        return float(np.median([r["ms"] for r in reps])), reps
+
+
+def combined_clocks(reps, max_mhz):
+    mhz = [r["sm_mhz"] for r in reps if r.get("sm_mhz")]
+    reasons = sorted({x for r in reps for x in r.get("reasons", [])})
+    return {"sm_mhz": float(np.median(mhz)) if mhz else None, "sm_max_mhz": max_mhz, "reasons": reasons,
+            "per_repeat_sm_mhz": mhz}
+
+
+def build_shards(args, w, N, rank, H, tables, batches):
+    """f3 at any N: table t -> S contiguous row shards, shard s on rank (owner[t] + s) % N.
+    Each rank needs the FULL CSR (global row ids) of every table it holds a shard of and the
+    rows of its shards; tables are generated (whole) on every rank that holds a shard."""
+    import torch
+    import synth.gpu as SG
+    S = args.shards
+    shards = []
+    for t in range(w.T):
+        cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(np.int64)
+        for sh in range(S):
+            shards.append((t, sh, int(cuts[sh]), int(cuts[sh + 1]), (int(w.owner[t]) + sh) % N))
+    mine = sorted((t, sh, lo, hi) for (t, sh, lo, hi, o) in shards if o == rank)
+    need = sorted({t for (t, _, _, _) in mine})
+    own_tables = list(w.local_tables(rank))
+    full = {}
+    for t in need:
+        full[t] = tables[own_tables.index(t)] if t in own_tables else SG.gen_table(w, int(w.phys[t]), int(w.rows[t]), H.dev)
+    shard_tabs = [full[t][lo:hi] for (t, sh, lo, hi) in mine]
+    # a workload view whose "local tables" are the tables with a local shard: its rank CSR
+    # is the full bag list of each such table (global ids), in ascending table order
+    wv = synth.make_workload(w.name, G=N, dist=w.dist, owner=np.array([rank if t in need else (rank + 1) % N
+                                                                          for t in range(w.T)]))
+
+    def shard_csr(seed):
+        off, idx = SG.rank_csr(wv, seed, rank, H.dev)
+        o_parts, x_parts, base = [torch.zeros(1, dtype=torch.int64, device=H.dev)], [], 0
+        for (t, sh, lo, hi) in mine:
+            tl = need.index(t)
+            seg = off[tl * w.B: (tl + 1) * w.B + 1]
+            o_parts.append(seg[1:] - seg[0] + base)
+            x_parts.append(idx[int(seg[0]): int(seg[-1])])
+            base += int(seg[-1] - seg[0])
+        return torch.cat(o_parts), torch.cat(x_parts) if x_parts else torch.zeros(0, dtype=torch.int64, device=H.dev)
+    new_batches = [shard_csr(w.batch_seed(i)) for i in range(len(batches))]
+    return shards, shard_tabs, new_batches, [t for (t, _, _, _) in mine], [(lo, hi) for (_, _, lo, hi) in mine]
+
+
+def run_backward(args, w, N, H, layer, batches, nnz, uniq, nbags, remote_bags):
     """One step = publish this rank's output-gradient slot + the fused backward kernel
     (one-sided loads of dY from the DP ranks, red.add into dW).  dY is synthetic
     (standard normal, filled once per slot, untimed); dW accumulates across steps."""
     import torch
-    import torch.distributed as dist
+    rank, dev, stream = H.rank, H.dev, H.stream
     dW = [torch.zeros((int(w.rows[t]), w.dim), device=dev) for t in w.local_tables(rank)]
     gen = torch.Generator(device=dev).manual_seed(1234 + rank)
     for _ in range(2):                                    # fill both ring slots once (untimed)
@@ -290,30 +436,31 @@ def run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq
 
     for s in range(args.warmup):
         bwd(s)
-    barrier()
-    with ClockSampler(local) as clk:
-        ms = timed(bwd, args.steps)
+    ms, reps = H.timed(bwd, args.steps, what="backward")
     assert layer.device_error() == 0, "device error during the timed region"
+    info = layer.info_now()
     value = w.B / (ms * 1e-3)
-    e, row = 4, w.dim * 4                                 # dW and dY are fp32
+    row = w.dim * 4                                       # dW and dY are fp32
     nnz_m, uniq_m = float(np.mean(nnz)), float(np.mean(uniq))
     lookup_bytes = nnz_m * (2 * row + 8) + nbags * (8 + row)      # row RMW per lookup + dY/offset per bag
     comp_bytes = uniq_m * 2 * row + nnz_m * 8 + nbags * (8 + row)  # each touched dW row read+written once
     nvl = remote_bags * row
     peak, peak_kind = hbm_peak()
-    t_hbm, t_nvl = comp_bytes / (peak * 1e9), nvl / (NVLINK_GBS * 1e9)
-    bound = "hbm" if t_hbm >= t_nvl else "nvlink"
+    t_roof = H.allreduce_max(max(comp_bytes / (peak * 1e9), nvl / (NVLINK_GBS * 1e9)))
+    bound = "hbm" if comp_bytes / peak >= nvl / NVLINK_GBS else "nvlink"
     ach = (comp_bytes if bound == "hbm" else nvl) / (ms * 1e-3) / 1e9
     pk = peak if bound == "hbm" else NVLINK_GBS
-    roof = {"bound": bound, "achieved": ach, "peak": pk, "unit": "GB/s", "frac": ach / pk, "traffic": None,
-            "kernel": "emb_bwd_kernel (one-sided dY loads + red.add.v4.f32 into dW)",
+    roof = {"bound": bound, "achieved": ach, "peak": pk, "unit": "GB/s", "frac": t_roof * 1e3 / ms, "traffic": None,
+            "traffic_source": None,
+            "kernel": "emb_bwd_kernel (one-sided dY loads + red.add.v4.f32 into dW)" if info["bwd_launches"] == 1 else
+                      "bwd_algo 1 pipeline (radix sort + segmented sum)",
             "algorithmic_bytes_per_launch": comp_bytes if bound == "hbm" else nvl,
             "basis": "compulsory: each touched dW row read+written once (2*d*4) + every index + every offset + "
-                     "every dY vector read once",
+                     "every dY vector read once; frac = max_r t_roof,r / max_r t_measured",
             "lookup_counted": {"bytes": lookup_bytes, "achieved": lookup_bytes / (ms * 1e-3) / 1e9,
                                "frac": lookup_bytes / (ms * 1e-3) / 1e9 / peak},
-            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs", "t_roof_ms": max(t_hbm, t_nvl) * 1e3}
-    if not args.opt:                                       # default kernel only: ncu of that kernel
+            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs", "t_roof_ms": t_roof * 1e3}
+    if not args.opt and args.shards == 1:                 # default kernel only: ncu of that kernel
         try:
             with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
                 tb = json.load(f).get(f"{w.name}:{w.dist}:G{N}:backward")
@@ -323,51 +470,39 @@ def run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq
         except (OSError, ValueError):
             pass
     layer.close()
+    # kernels per step: the backward path, + at N > 1 the slot-wait and the ready-signal kernels
+    launches = args.steps * (info["bwd_launches"] + (2 if N > 1 else 0))
     if N > 1:
-        dist.barrier()
-    if rank == 0:
+        H.dist.barrier()
+    if H.rank == 0:
         line = {"metric": "EMB bwd samples/sec (max over ranks)", "value": value, "unit": "samples/s", "n_gpus": N,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "steps": args.steps, "warmup": args.warmup, "repeats": len(reps), "ms_per_step": ms,
+                "ms_per_step_repeats": [r["ms"] for r in reps], "higher_is_better": True,
                 "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic", "config": {**config_desc(w, N), "mode": "backward (SURVEY f2)"},
-                "roofline": roof, "cpu_baseline": None, "e2e": None, "gpu_launches": args.steps * (2 if N > 1 else 1),
-                "clocks": clk.summary()}
+                "data": "synthetic", "config": {**config_desc(w, N, args), "mode": "backward (SURVEY f2)"},
+                "roofline": roof, "cpu_baseline": None, "e2e": None, "gpu_launches": launches,
+                "clocks": combined_clocks(reps, ClockSampler(H.local).max_mhz)}
         print(json.dumps(line), flush=True)
     if N > 1:
-        dist.destroy_process_group()
+        H.dist.destroy_process_group()
     return 0
 
 
-# ------------------------------------------------------------------------------ GPU arm
 def main():
     args = parse()
     if args.impl == "reference":
         return reference_arm(args)
     import torch
-    import torch.distributed as dist
 
     from paper_conf_sc_chenbyo24_b200 import emb as E
     from paper_conf_sc_chenbyo24_b200.comm import torch_allgather
     from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
     import synth.gpu as SG
 
-    N = args.gpus
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world != N:
-        raise SystemExit(f"--gpus {N} but WORLD_SIZE={world}")
-    if args.same_device:
-        local = 0
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    if N > 1:
-        if args.backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:
-            dist.init_process_group("gloo")
+    H = Harness(args)
+    N, rank, dev, stream = H.N, H.rank, H.dev, H.stream
     w = synth.make_workload(args.config, G=N, dist=args.dist)
-    stream = torch.cuda.Stream(device=dev)
+    ib = args.index_bits // 8
 
     # ---- inputs in HBM (untimed)
     with torch.cuda.stream(stream):
@@ -378,125 +513,106 @@ def main():
     for kv in args.opt:
         k, v = kv.split("=")
         opts[k] = int(v)
-    nnz = [int(b[0][-1].item()) for b in batches]
-    uniq = [unique_rows(w, rank, b) for b in batches]     # untimed: compulsory-traffic basis
-    w._shards = args.shards
     shards = None
+    stat_tables = list(w.local_tables(rank))              # tables whose full CSR this rank reads
+    ranges = None                                         # f3: row range of each local shard
     if args.shards > 1:
-        # f3: table t -> S row shards, shard s on rank (owner[t] + s) % N; each rank needs the
-        # FULL CSR of every table it holds a shard of.  Tables are generated where the
-        # table's owner is; at N = 1 every shard is a view of the local table.
-        if N > 1:
-            raise SystemExit("--shards > 1 is exercised at N = 1 in this round (all shards local)")
+        if args.mode == "backward":
+            raise SystemExit("--shards > 1 has no backward (f2 is table-wise)")
         args.no_control = True       # the uniform control and the comparison path are table-wise
         args.no_compare = True
-        S = args.shards
-        shards = []
-        for t in range(w.T):
-            cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(np.int64)
-            for sh in range(S):
-                shards.append((t, sh, int(cuts[sh]), int(cuts[sh + 1]), (int(w.owner[t]) + sh) % N))
-        tables = [tables[list(w.local_tables(rank)).index(t)][lo:hi] for (t, sh, lo, hi, o) in sorted(shards)]
-
-        def shard_csr(batch):
-            off, idx = batch
-            lt = list(w.local_tables(rank))
-            o_parts, x_parts, base = [torch.zeros(1, dtype=torch.int64, device=dev)], [], 0
-            for (t, sh, lo, hi, o) in sorted(shards):
-                tl = lt.index(t)
-                seg = off[tl * w.B: (tl + 1) * w.B + 1]
-                o_parts.append(seg[1:] - seg[0] + base)
-                x_parts.append(idx[int(seg[0]): int(seg[-1])])
-                base += int(seg[-1] - seg[0])
-            return torch.cat(o_parts), torch.cat(x_parts)
-        batches = [shard_csr(b) for b in batches]
+        shards, tables, batches, stat_tables, ranges = build_shards(args, w, N, rank, H, tables, batches)
         torch.cuda.synchronize()
-    layer = PgasEmbedding(rank, N, local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
+    nnz = [int(b[0][-1].item()) for b in batches]
+    uniq = [unique_rows(w, stat_tables, b, ranges) for b in batches]     # untimed: compulsory-traffic basis
+    if ib == 4:
+        batches = [(o.to(torch.int32), x.to(torch.int32)) for o, x in batches]
+        torch.cuda.synchronize()
+    layer = PgasEmbedding(rank, N, H.local, w.rows, w.owner, w.dim, tables, w.B, w.wdtype, w.odtype,
                           torch_allgather() if N > 1 else None, opts, backward=(args.mode == "backward"),
                           shards=shards)
     T_r = len(w.local_tables(rank))
-    nbags = T_r * w.B
+    nbags = len(stat_tables) * w.B
     B_r = layer.B_r
-    remote_bags = T_r * (w.B - B_r)
+    # NVLink bytes of this rank's one-sided stores (egress) and of the stores it receives
+    eo_row = w.dim * (4 if shards is not None else w.out_elem_bytes())     # f3 partials are fp32
+    egress = len(stat_tables) * (w.B - B_r) * eo_row
+    ingress = (len(shards) - len(stat_tables) if shards is not None else (w.T - T_r)) * B_r * eo_row
 
-    def barrier():
-        if N > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-
-    def timed(fn, steps, finish=None):
-        barrier()
-        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ev0.record(stream)
-        for s in range(steps):
-            fn(s)
-        if finish is not None:
-            finish()
-        ev1.record(stream)
-        torch.cuda.synchronize()
-        ms = ev0.elapsed_time(ev1) / steps
-        if N > 1:
-            t = torch.tensor([ms], device=dev if args.backend == "nccl" else "cpu")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = float(t.item())
-        return ms
+    if args.mode == "backward":
+        return run_backward(args, w, N, H, layer, batches, nnz, uniq, nbags, T_r * (w.B - B_r))
 
     def fwd(s):
         o, x = batches[s % len(batches)]
         layer.forward(o, x, 0, stream)
 
-    if args.mode == "backward":
-        return run_backward(args, w, N, rank, local, dev, stream, layer, batches, nnz, uniq, nbags, remote_bags,
-                            barrier, timed)
-
     for s in range(args.warmup):
         fwd(s)
-    barrier()
-    with ClockSampler(local) as clk:
-        ms = timed(fwd, args.steps)
+    ms, reps = H.timed(fwd, args.steps)
     assert layer.device_error() == 0, "device error during the timed region"
     value = w.B / (ms * 1e-3)
+    info = layer.info_now()
 
-    lookup_bytes, nvl_bytes = algorithmic_bytes(w, float(np.mean(nnz)), nbags, remote_bags)
-    hbm_bytes = float(np.mean([compulsory_bytes(w, u, z, nbags) for u, z in zip(uniq, nnz)]))
+    lookup_bytes = algorithmic_bytes(w, float(np.mean(nnz)), nbags, ib)
+    hbm_bytes = float(np.mean([compulsory_bytes(w, u, z, nbags, ib) for u, z in zip(uniq, nnz)]))
     peak, peak_kind = hbm_peak()
     t_hbm = hbm_bytes / (peak * 1e9)
-    t_nvl = nvl_bytes / (NVLINK_GBS * 1e9)
-    bound = "hbm" if t_hbm >= t_nvl else "nvlink"
-    achieved = (hbm_bytes if bound == "hbm" else nvl_bytes) / (ms * 1e-3) / 1e9
+    t_nvl = max(egress, ingress) / (NVLINK_GBS * 1e9)
+    t_roof_r = max(t_hbm, t_nvl)
+    t_roof = H.allreduce_max(t_roof_r)                    # max_r t_roof,r / max_r t_measured,r
+    per_rank = H.gather({"rank": rank, "t_roof_ms": t_roof_r * 1e3, "hbm_compulsory_bytes": hbm_bytes,
+                         "lookup_bytes": lookup_bytes, "nvlink_egress_bytes": egress, "nvlink_ingress_bytes": ingress,
+                         "unique_rows": float(np.mean(uniq)), "lookups": float(np.mean(nnz))})
+    binding = max(per_rank, key=lambda d: d["t_roof_ms"])
+    b_hbm = binding["hbm_compulsory_bytes"] / (peak * 1e9)
+    b_nvl = max(binding["nvlink_egress_bytes"], binding["nvlink_ingress_bytes"]) / (NVLINK_GBS * 1e9)
+    bound = "hbm" if b_hbm >= b_nvl else "nvlink"
+    bytes_bound = binding["hbm_compulsory_bytes"] if bound == "hbm" else max(binding["nvlink_egress_bytes"],
+                                                                              binding["nvlink_ingress_bytes"])
     pk = peak if bound == "hbm" else NVLINK_GBS
-    traffic = None
-    l2 = None
-    try:
-        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            tj = json.load(f)
-        key = f"{w.name}:{w.dist}:G{N}"  # profiles/traffic.json: ncu --set full of this workload
-        if key in tj:
-            traffic = tj[key]["dram_bytes_per_launch"]
-            with open(os.path.join(ROOT, "profiles", "l2_probe.json")) as f:
-                l2_peak = float(json.load(f)["l2_read_peak_gbs"])
-            l2_bytes = tj[key].get("l2_read_bytes_per_launch")
-            if l2_bytes:
-                # second roof: L2->SM read traffic of this kernel (ncu) over the measured L2
-                # streaming read bandwidth (tools/l2_probe.py); binds under zipf reuse
-                l2 = {"bytes": l2_bytes, "achieved": l2_bytes / (ms * 1e-3) / 1e9, "peak": l2_peak, "unit": "GB/s",
-                      "frac": l2_bytes / (ms * 1e-3) / 1e9 / l2_peak,
-                      "source": "ncu lts__t_sectors_srcunit_tex_op_read x 32 B (profiles/traffic.json) / "
-                                "profiles/l2_probe.json"}
-    except Exception:
-        pass
-    roof = {"bound": bound, "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": achieved / pk,
-            "traffic": traffic, "kernel": "emb_fwd_kernel (fused gather+pool+store+flags)",
-            "algorithmic_bytes_per_launch": hbm_bytes if bound == "hbm" else nvl_bytes,
-            "basis": "compulsory HBM bytes: each distinct (table,row) of the batch once (d*e) + every index (8 B) "
-                     "+ every offset (8 B) + every pooled output vector written once (d*e_o); SURVEY §8(d) fraction 3",
+    achieved = bytes_bound / (ms * 1e-3) / 1e9
+    default_kernel = not args.opt and args.shards == 1 and ib == 8
+    traffic, traffic_src, l2 = None, None, None
+    if default_kernel:                                    # the committed ncu capture is of the default kernel
+        try:
+            with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+                tj = json.load(f)
+            key = f"{w.name}:{w.dist}:G{N}"  # profiles/traffic.json: ncu --set full of this workload
+            if key in tj:
+                traffic = tj[key]["dram_bytes_per_launch"]
+                traffic_src = tj[key].get("source")
+                with open(os.path.join(ROOT, "profiles", "l2_probe.json")) as f:
+                    l2_peak = float(json.load(f)["l2_read_peak_gbs"])
+                l2_bytes = tj[key].get("l2_read_bytes_per_launch")
+                if l2_bytes:
+                    # second roof: L2->SM read traffic of this kernel (ncu) over the measured L2
+                    # read bandwidth of the same gather on an L2-resident table
+                    l2 = {"bytes": l2_bytes, "achieved": l2_bytes / (ms * 1e-3) / 1e9, "peak": l2_peak,
+                          "unit": "GB/s", "frac": l2_bytes / (ms * 1e-3) / 1e9 / l2_peak,
+                          "source": "ncu lts__t_sectors_srcunit_tex_op_read x 32 B (profiles/traffic.json) / "
+                                    "profiles/l2_probe.json"}
+        except Exception:
+            pass
+    roof = {"bound": bound, "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": t_roof * 1e3 / ms,
+            "traffic": traffic, "traffic_source": traffic_src if traffic is not None else
+            ("no ncu capture of this variant" if not default_kernel else "no capture of this workload"),
+            "kernel": "emb_fwd_kernel (fused gather+pool+store+flags)",
+            "algorithmic_bytes_per_launch": bytes_bound,
+            "basis": "compulsory HBM bytes: each distinct (table,row) of the batch once (d*e) + every index + "
+                     "every offset + every pooled output vector written once (d*e_o); NVLink: max(egress, ingress) "
+                     "of the one-sided stores; frac = max_r t_roof,r / max_r t_measured (SURVEY §8(d))",
             "lookup_counted": {"bytes": lookup_bytes, "achieved": lookup_bytes / (ms * 1e-3) / 1e9,
                                "frac": lookup_bytes / (ms * 1e-3) / 1e9 / peak,
                                "note": "every lookup's row counted (SURVEY §8(d) fraction 1); >1 under zipf "
                                        "because L1/L2 serve repeated rows"},
             "unique_rows_per_batch": float(np.mean(uniq)), "lookups_per_batch": float(np.mean(nnz)),
-            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else "measured peer copy 770 GB/s (B200_PROFILING.md)",
-            "t_roof_ms": max(t_hbm, t_nvl) * 1e3, "frac_of_roofline_time": max(t_hbm, t_nvl) * 1e3 / ms,
+            "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else
+                           "measured peer copy 770 GB/s (B200_PROFILING.md)",
+            "t_roof_ms": t_roof * 1e3, "binding_rank": binding["rank"], "per_rank": per_rank,
+            "nvlink": {"egress_bytes_max": max(d["nvlink_egress_bytes"] for d in per_rank),
+                       "ingress_bytes_max": max(d["nvlink_ingress_bytes"] for d in per_rank),
+                       "achieved_gbs": max(d["nvlink_egress_bytes"] for d in per_rank) / (ms * 1e-3) / 1e9,
+                       "peak": NVLINK_GBS, "peak_nominal": 900.0},
             "l2": l2}
 
     extra = {}
@@ -506,36 +622,81 @@ def main():
         with torch.cuda.stream(stream):
             ub = [SG.rank_csr(wu, wu.batch_seed(100 + i), rank, dev) for i in range(2)]
         torch.cuda.synchronize()
+        nnz_u = [int(b[0][-1].item()) for b in ub]
+        cb_u = float(np.mean([compulsory_bytes(wu, unique_rows(wu, stat_tables, b), z, nbags, ib)
+                              for b, z in zip(ub, nnz_u)]))
+        if ib == 4:
+            ub = [(o.to(torch.int32), x.to(torch.int32)) for o, x in ub]
         for s in range(3):
             layer.forward(ub[s % 2][0], ub[s % 2][1], 0, stream)
 
         def fwd_u(s):
             layer.forward(ub[s % 2][0], ub[s % 2][1], 0, stream)
-        ms_u = timed(fwd_u, max(args.steps // 2, 3))
-        nnz_u = [int(b[0][-1].item()) for b in ub]
-        hb_u, _ = algorithmic_bytes(wu, float(np.mean(nnz_u)), nbags, remote_bags)
-        cb_u = float(np.mean([compulsory_bytes(wu, unique_rows(wu, rank, b), z, nbags) for b, z in zip(ub, nnz_u)]))
+        ms_u, _ = H.timed(fwd_u, max(args.steps // 2, 3), what="uniform_control")
+        t_roof_u = H.allreduce_max(max(cb_u / (peak * 1e9), t_nvl))
+        hb_u = algorithmic_bytes(wu, float(np.mean(nnz_u)), nbags, ib)
         extra["uniform_control"] = {"ms_per_step": ms_u, "value": w.B / (ms_u * 1e-3),
-                                    "achieved_gbs": cb_u / (ms_u * 1e-3) / 1e9, "frac": cb_u / (ms_u * 1e-3) / 1e9 / peak,
+                                    "achieved_gbs": cb_u / (ms_u * 1e-3) / 1e9, "frac": t_roof_u * 1e3 / ms_u,
                                     "lookup_counted_frac": hb_u / (ms_u * 1e-3) / 1e9 / peak,
                                     "note": "uniform indices: lookup-counted ~= compulsory ~= DRAM bytes"}
         del ub
 
-    # ---- conventional comparison path: pool kernel -> NCCL all_to_all_single -> unpack kernel
+    # ---- conventional comparison path: pool kernel -> NCCL all_to_all_single -> unpack kernel,
+    # with the paper's time breakdown (§IV-A-2a; Figs. 6/9): the exchange
+    # phase (a2a + wait + unpack) measured with the full volume and again sending ONE float
+    # per peer; Sync+Unpack := the one-float phase (over-estimated by one float's latency),
+    # Communication := full phase - one-float phase (under-estimated: latency excluded),
+    # Computation := the pool kernel alone.
     if not args.no_compare:
-        def fwd_b(s):
-            o, x = batches[s % len(batches)]
-            with torch.cuda.stream(stream):
-                layer.forward_baseline(o, x, None, 0, stream)
+        def run_b(single, pool_only=False):
+            def f(s):
+                o, x = batches[s % len(batches)]
+                with torch.cuda.stream(stream):
+                    layer.forward_baseline(o, x, None, 0, stream, single_float=single, pool_only=pool_only)
+            return f
         for s in range(3):
-            fwd_b(s)
-        ms_b = timed(fwd_b, max(args.steps // 2, 3))
-        extra["comparison_nccl_path"] = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3),
-                                         "pgas_speedup": ms_b / ms,
-                                         "note": "G=1: pool kernel only (no exchange, no unpack)" if N == 1 else
-                                         f"pool kernel + {args.backend} all_to_all_single + unpack kernel"
-                                         + (" (gloo: host-staged test harness, not a measurement)"
-                                            if args.backend == "gloo" else "")}
+            run_b(False)(s)
+        k_b = max(args.steps // 2, 3)
+        ms_b, _ = H.timed(run_b(False), k_b, what="nccl_path")
+        cmp = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3), "pgas_speedup": ms_b / ms}
+        if N == 1:
+            cmp["note"] = "G=1: pool kernel only (no exchange, no unpack)"
+            cmp["breakdown"] = {"computation_ms": ms_b, "communication_ms": 0.0, "sync_unpack_ms": 0.0}
+        else:
+            for s in range(3):
+                run_b(True)(s)
+            ms_1, _ = H.timed(run_b(True), k_b, what="nccl_path_one_float")
+            ms_p, _ = H.timed(run_b(False, pool_only=True), k_b, what="nccl_path_pool_only")
+            phase, phase1 = ms_b - ms_p, ms_1 - ms_p
+            cmp["note"] = f"pool kernel + {args.backend} all_to_all_single(async_op=True).wait() + unpack kernel" + \
+                (" (gloo: host-staged test harness, not a measurement)" if args.backend == "gloo" else "")
+            cmp["breakdown"] = {"computation_ms": ms_p, "communication_ms": max(phase - phase1, 0.0),
+                                "sync_unpack_ms": phase1, "exchange_phase_ms": phase,
+                                "exchange_phase_one_float_ms": phase1,
+                                "method": "PAPER.md L286-292: phase (a2a + wait + unpack) timed with the full volume "
+                                          "and with one float per peer; sync+unpack = one-float phase, "
+                                          "communication = full - one-float; computation = pool kernel alone"}
+        extra["comparison_nccl_path"] = cmp
+
+    # ---- f1: per-rank communication timeline of one traced forward (not timed)
+    if not args.no_trace:
+        E.emb_set_option(layer.ctx, "trace_capacity", 1 << 21)
+        for s in range(2):
+            E.emb_trace_read(layer.ctx, 0)
+            H.barrier()
+            fwd(s)
+            torch.cuda.synchronize()
+        summ = trace_summary(E.emb_trace_read(layer.ctx, 1 << 21))
+        E.emb_set_option(layer.ctx, "trace_capacity", 0)
+        allsum = H.gather(summ)
+        t0 = min(s.get("t0_ns", 1 << 62) for s in allsum)
+        for r, s in enumerate(allsum):
+            s["rank"] = r
+            if "t0_ns" in s:
+                s["start_offset_us"] = (s.pop("t0_ns") - t0) / 1e3
+        extra["comm_timeline"] = {"per_rank": allsum, "bins": 40,
+                                  "note": "f1 (PAPER.md L294, Figs. 7/10): per-chunk {globaltimer, bytes stored to "
+                                          "peers / locally} of one traced forward, binned over each rank's span"}
 
     # ---- e2e through the public C ABI with host buffers
     e2e = None
@@ -555,36 +716,40 @@ def main():
             fwd_h(s)
         drain()
         k_e2e = max(min(args.steps, 20), 3)
-        ms_e = timed(fwd_h, k_e2e, drain)
-        h2d = float(np.mean([(ho.numel() + hx.numel()) * 8 for ho, hx in hb]))
+        ms_e, _ = H.timed(fwd_h, k_e2e, drain, what="e2e")
+        h2d = float(np.mean([(ho.numel() + hx.numel()) * ib for ho, hx in hb]))
         d2h = B_r * w.T * w.dim * w.out_elem_bytes()
         e2e = {"value": w.B / (ms_e * 1e-3), "unit": "samples/s", "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": ms_e, "steps": k_e2e,
-               "path": "emb_forward_host_async (public C ABI): pinned H2D of offsets+indices on a copy-in stream, "
-                       "fused kernel on the caller's stream, D2H of Y_r on a copy-out stream; consecutive steps "
-                       "overlap; the timed region ends after emb_host_drain"}
+               "path": ("emb_forward_host_async_i32" if ib == 4 else "emb_forward_host_async") +
+                       " (public C ABI): pinned H2D of offsets+indices on a copy-in stream, fused kernel on the "
+                       "caller's stream, D2H of Y_r on a copy-out stream; consecutive steps overlap; the timed "
+                       "region ends after emb_host_drain"}
 
     cpu = None
-    if rank == 0 and N == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:
         cpu = oracle_sample(w, 0)
-
+        cpu["rank"] = 0
     layer.close()
     if N > 1:
-        dist.barrier()
+        H.dist.barrier()
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "steps": args.steps, "warmup": args.warmup, "repeats": len(reps), "ms_per_step": ms,
+                "ms_per_step_repeats": [r["ms"] for r in reps], "higher_is_better": True,
                 "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None,
                 "dtype": "f32" if (w.wdtype == "f32") else "bf16", "data": "synthetic",
-                "config": config_desc(w, N), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "config": config_desc(w, N, args), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
                 "pooled_vectors_per_s": w.B * w.T / (ms * 1e-3),
                 "scaling_note": "table-wise model parallelism: each GPU adds its tables AND (weak) its 16,384 samples, so "
                                 "every GPU pools its tables for the whole global batch; ideal samples/s is flat in N, "
                                 "pooled_vectors_per_s (samples x tables) is the quantity that ideally grows with N",
-                "gpu_launches": args.steps, "clocks": clk.summary(), **extra}
+                "gpu_launches": args.steps * info["fwd_launches"],
+                "clocks": combined_clocks(reps, ClockSampler(H.local).max_mhz),
+                "clock_log": H.clock_log, **extra}
         print(json.dumps(line), flush=True)
     if N > 1:
-        dist.destroy_process_group()
+        H.dist.destroy_process_group()
     return 0
 
 

@@ -22,13 +22,17 @@ Readings of points the paper leaves open (listed in DESIGN.md "Readings"):
   accumulator starts at the FIRST row, then float32 round-to-nearest adds;
   C5  float32 accumulation (also for bf16 tables, widened exactly);
   C6  bf16 output = RNE of the float32 accumulator, once;
+  C7  IEEE arithmetic without flush-to-zero (numpy float32 adds keep subnormals); Inf and
+      NaN propagate; NaN -> NaN in the bf16 rounding;
   C8  contiguous batch split, first B mod G ranks one extra sample;
   C9  output [B_r][T][d] row-major, tables in global id order;
   C11 per-rank CSR is table-major: bag (t_l, b) = offsets[t_l*B+b] .. offsets[t_l*B+b+1];
   C13 duplicate indices all count.
 
 Pins (tests/test_oracle.py): brute-force Python loops (P1), one-hot/empty/duplicate
-closed forms (P2-P4), integer tables exact in any order (P5), identity routing (P6),
+closed forms (P2-P4), the S-normalised metric and S = sum |w| against hand-derived values
+(tests/golden/s_normalized_error.json), IEEE special values (subnormal sums, +-Inf, NaN;
+C7) against closed forms and torch's bf16 conversion, integer tables exact in any order (P5), identity routing (P6),
 power-of-two scaling (P7), linearity (P8), placement invariance (P9), rank concat
 (P10), torch.nn.functional.embedding_bag + gloo all_to_all special cases (P11),
 conservation (P13), the paper's Fig. 3 / Fig. 4 structure (P15), and torch's bf16
@@ -130,10 +134,16 @@ def pool_bag_f64(rows: np.ndarray) -> Tuple[np.ndarray, np.ndarray]:
 # ----------------------------------------------------------------------------- bf16
 def rne_bf16(x: np.ndarray) -> np.ndarray:
     """float32 -> bf16 bits, round to nearest even (C6): u += 0x7FFF + ((u>>16)&1); u >>= 16.
-    (Inputs are finite; NaN handling is not needed by the generators, C7.)"""
-    u = np.ascontiguousarray(x, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    Finite values overflow to +-Inf and subnormals round like any other value (the rule is
+    monotone in the bit pattern); +-Inf map to +-Inf.  NaN stays NaN (C7): the rounding rule
+    would carry a NaN whose payload sits in the low 16 bits into Inf, so NaN is mapped to
+    the quiet NaN 0x7FC0 instead (any NaN pattern is accepted on the GPU side)."""
+    f = np.ascontiguousarray(x, dtype=np.float32)
+    u = f.view(np.uint32).astype(np.uint64)
     u = u + np.uint64(0x7FFF) + ((u >> np.uint64(16)) & np.uint64(1))
-    return (u >> np.uint64(16)).astype(np.uint16)
+    out = (u >> np.uint64(16)).astype(np.uint16)
+    out[np.isnan(f)] = np.uint16(0x7FC0)
+    return out
 
 
 def bf16_to_f32(bits: np.ndarray) -> np.ndarray:

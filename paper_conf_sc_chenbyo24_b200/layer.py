@@ -80,24 +80,36 @@ class PgasEmbedding:
         return self._send, self._recv, self._out
 
     def forward_baseline(self, offsets: torch.Tensor, indices: torch.Tensor, group=None, flags: int = 0,
-                         stream=None) -> torch.Tensor:
+                         stream=None, single_float: bool = False, pool_only: bool = False) -> torch.Tensor:
+        """pool kernel -> all_to_all_single(async_op=True).wait() -> unpack kernel (L155, L193).
+        single_float: the exchange sends ONE float per peer instead of the pooled vectors and the
+        unpack still runs over the (stale) receive buffer -- the paper's probe for the
+        sync + unpack share of the exchange phase (L286-292); pool_only: stop after the pool."""
         send, recv, out = self._baseline_buffers()
         E.emb_baseline_pool(self.ctx, offsets, indices, send, flags, stream)
-        if self.ctx.world_size == 1:  # G = 1: send already is [B][T][d]; no exchange, no unpack
+        if self.ctx.world_size == 1 or pool_only:  # G = 1: send already is [B][T][d]; no exchange, no unpack
             return send[: self.B_r * self.T * self.dim].view(self.B_r, self.T, self.dim)
         import torch.distributed as dist
+        G = self.ctx.world_size
+        sc, rc = self._send_counts, self._recv_counts
+        s_in, s_out = (send, recv) if not single_float else (send[:G], recv[:G])
+        if single_float:
+            sc, rc = [1] * G, [1] * G
         if dist.get_backend(group) == "nccl":
-            work = dist.all_to_all_single(recv, send, output_split_sizes=self._recv_counts,
-                                          input_split_sizes=self._send_counts, group=group, async_op=True)
+            work = dist.all_to_all_single(s_out, s_in, output_split_sizes=rc, input_split_sizes=sc, group=group,
+                                          async_op=True)
             work.wait()
         else:  # gloo (CPU test harness): stage the exchange through host memory
             torch.cuda.current_stream(self.device).synchronize() if stream is None else stream.synchronize()
-            hs, hr = send.cpu(), torch.empty(recv.shape, dtype=recv.dtype)
-            dist.all_to_all_single(hr, hs, output_split_sizes=self._recv_counts,
-                                   input_split_sizes=self._send_counts, group=group)
-            recv.copy_(hr)
+            hs, hr = s_in.cpu(), torch.empty(s_out.shape, dtype=s_out.dtype)
+            dist.all_to_all_single(hr, hs, output_split_sizes=rc, input_split_sizes=sc, group=group)
+            s_out.copy_(hr)
         E.emb_baseline_unpack(self.ctx, recv, out, stream)
         return out
+
+    def info_now(self) -> dict:
+        """emb_get_info of the context (epoch, launch shape, kernels per call, ...)."""
+        return E.emb_get_info(self.ctx)
 
     # ---- f2 backward (PAPER.md §V L378-382) ---------------------------------------------
     def grad_slot(self, stream=None) -> torch.Tensor:

@@ -30,6 +30,9 @@ def test_bench_n1_contract():
     d = _last_json(r.stdout)
     assert KEYS <= set(d), KEYS - set(d)
     assert d["n_gpus"] == 1 and d["steps"] == 5 and d["gpu_launches"] == 5 and d["value"] > 0
+    assert d["repeats"] == 5 and len(d["ms_per_step_repeats"]) == 5
+    assert d["ms_per_step"] == sorted(d["ms_per_step_repeats"])[2]               # the median repeat
+    assert len(d["clocks"]["per_repeat_sm_mhz"]) <= 5
     assert d["roofline"]["bound"] in ("hbm", "nvlink") and d["roofline"]["peak"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
@@ -45,10 +48,40 @@ def test_bench_reference_arm():
 
 
 def test_bench_two_ranks_one_gpu():
+    """The driver's N > 1 line, produced by 2 ranks time-slicing one GPU (gloo harness):
+    cpu_baseline present, roofline from max_r t_roof over per-rank bytes, the paper's
+    compute / communication / sync+unpack breakdown of the comparison path, and a per-rank
+    f1 communication timeline."""
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
            "127.0.0.1", "--master-port", "29561", "bench.py", "--gpus", "2", "--steps", "5", "--warmup", "3",
-           "--config", "tiny", "--backend", "gloo", "--same-device", "--no-cpu-baseline"]
+           "--config", "tiny", "--backend", "gloo", "--same-device", "--repeats", "3"]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-3000:]
     d = _last_json(r.stdout)
-    assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["global_batch"] == 32
+    assert KEYS <= set(d), KEYS - set(d)
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["global_batch"] == 32 and d["repeats"] == 3
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] > 0
+    roof = d["roofline"]
+    assert len(roof["per_rank"]) == 2 and roof["binding_rank"] in (0, 1)
+    assert abs(roof["t_roof_ms"] - max(p["t_roof_ms"] for p in roof["per_rank"])) < 1e-9
+    assert abs(roof["frac"] - roof["t_roof_ms"] / d["ms_per_step"]) < 1e-9
+    assert roof["nvlink"]["egress_bytes_max"] > 0
+    bd = d["comparison_nccl_path"]["breakdown"]
+    assert {"computation_ms", "communication_ms", "sync_unpack_ms", "exchange_phase_ms"} <= set(bd)
+    tl = d["comm_timeline"]["per_rank"]
+    assert len(tl) == 2 and all(t["records"] > 0 and t["remote_bytes"] > 0 for t in tl)
+    assert d["e2e"]["h2d_bytes_per_step"] > 0
+
+
+def test_bench_int32_and_shards_lines():
+    """--index-bits 32 (C12 option) and --shards 2 (f3) produce complete lines at N = 1;
+    their roofline carries no ncu traffic of the default kernel."""
+    for extra in (["--index-bits", "32"], ["--shards", "2"]):
+        r = subprocess.run([sys.executable, "bench.py", "--config", "tiny", "--steps", "5", "--warmup", "3",
+                            "--repeats", "2", "--no-cpu-baseline", *extra], cwd=ROOT, capture_output=True, text=True,
+                           timeout=600)
+        assert r.returncode == 0, r.stderr[-3000:]
+        d = _last_json(r.stdout)
+        assert d["value"] > 0 and d["roofline"]["traffic"] is None
+        if extra[0] == "--index-bits":
+            assert d["config"]["index_bits"] == 32 and "i32" in d["e2e"]["path"]

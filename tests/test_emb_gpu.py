@@ -416,3 +416,78 @@ def test_trace_counts_every_stored_byte():
         assert E.emb_trace_read(layers[0].ctx, 10).shape[0] == 0
     finally:
         _close(layers)
+
+
+def _c7_tables(w, seed):
+    """Tables of IEEE special values (SURVEY reading C7: IEEE RN, no FTZ, NaN propagates):
+    table 0 holds only small multiples of the least subnormal (its bag sums stay subnormal,
+    an FTZ add would return 0) and -0.0; table 1 normal values sprinkled with +-Inf, NaN and
+    near-max finites (sums overflow to Inf, Inf - Inf = NaN); table 2 large-magnitude
+    cancellation (+-2^100 against O(1) values) and -0.0 rows.  All values are exact in the
+    weight dtype (bf16 tables: multiples of 2^-133, quiet NaN 0x7FC00000)."""
+    rng = np.random.default_rng(seed)
+    M, d = int(w.rows[0]), w.dim
+    bf = w.wdtype == "bf16"
+    lsb = 2.0 ** (-133 if bf else -149)
+    out = {}
+    t0 = (rng.integers(-40, 41, size=(M, d)) * lsb).astype(np.float32)
+    t0[rng.random((M, d)) < 0.1] = -0.0
+    out[0] = t0
+    t1 = (rng.integers(-128, 128, size=(M, d)) / 64.0).astype(np.float32)
+    u = rng.random((M, d))
+    big = np.float32(2.0 ** 127 * 1.5)                       # exact in bf16, two of them overflow
+    t1[u < 0.02] = np.inf
+    t1[(u >= 0.02) & (u < 0.04)] = -np.inf
+    t1[(u >= 0.04) & (u < 0.06)] = np.uint32(0x7FC00000).view(np.float32)
+    t1[(u >= 0.06) & (u < 0.08)] = big
+    t1[(u >= 0.08) & (u < 0.10)] = -big
+    out[1] = t1
+    t2 = (rng.integers(-8, 9, size=(M, d)) / 4.0).astype(np.float32)
+    v = rng.random((M, d))
+    t2[v < 0.15] = np.float32(2.0 ** 100)
+    t2[(v >= 0.15) & (v < 0.30)] = np.float32(-(2.0 ** 100))
+    t2[rng.random(M) < 0.1] = -0.0
+    out[2] = t2
+    return out
+
+
+def _assert_ieee_equal(got, ref):
+    """bit-exact, except that a NaN matches any NaN (its payload is not specified, C7)"""
+    gf = got.astype(np.float32) if got.dtype == np.float32 else O.bf16_to_f32(got)
+    rf = ref.astype(np.float32) if ref.dtype == np.float32 else O.bf16_to_f32(ref)
+    gn, rn = np.isnan(gf), np.isnan(rf)
+    assert np.array_equal(gn, rn), f"NaN positions differ: {np.argwhere(gn != rn)[:3].tolist()}"
+    gb, rb = H.bits(got), H.bits(ref)
+    bad = (gb != rb) & ~gn
+    assert not bad.any(), f"{int(bad.sum())} mismatches, first at {np.argwhere(bad)[0].tolist()}: " \
+                          f"got {gf[tuple(np.argwhere(bad)[0])]!r} want {rf[tuple(np.argwhere(bad)[0])]!r}"
+
+
+@pytest.mark.parametrize("dim,wdt,odt", [(128, "f32", "f32"), (64, "f32", "f32"), (256, "bf16", "bf16"),
+                                         (128, "bf16", "f32"), (64, "f32", "bf16")])
+@pytest.mark.parametrize("G", [1, 2])
+def test_c7_ieee_special_values_bitexact(dim, wdt, odt, G):
+    """C7 on the GPU: subnormal sums are not flushed, +-Inf / NaN propagate, overflow gives
+    Inf, -0.0 one-hot bags keep their sign, large-magnitude cancellation follows the
+    canonical order -- bit-exact against the oracle (NaN matched as NaN), through the
+    direct kernel, the per-id validity kernel (CHECK_BOUNDS) and, at G = 2, remote stores."""
+    w = synth.make_workload("tiny", G=G, T=3, rows=64, dim=dim, B=203, pmin=0, pmax=12, wdtype=wdt, odtype=odt)
+    tabs = _c7_tables(w, 17)
+    csr = H.np_csrs(w, 19)
+    with np.errstate(all="ignore"):
+        ref = H.oracle_outputs(w, 19, tabs, csr)
+    r0 = ref[0].astype(np.float32) if ref[0].dtype == np.float32 else O.bf16_to_f32(ref[0])
+    assert np.isnan(r0).any() and np.isinf(r0).any()                      # the specials do reach the output
+    if G == 1 and (odt == "f32" or wdt == "bf16"):
+        sub = r0[:, 0]
+        assert ((sub != 0) & (np.abs(sub) < 2.0 ** -126)).any()            # subnormal results present
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, csr)
+        got_chk = _run(w, layers, csr, E.EMB_FWD_CHECK_BOUNDS)
+        for r in range(w.G):
+            _assert_ieee_equal(got[r], ref[r])
+            _assert_ieee_equal(got_chk[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)

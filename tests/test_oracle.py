@@ -483,3 +483,78 @@ def test_f3_shard_order_sum_and_tolerance():
             for p_ in parts[1:]:
                 acc = acc + p_
             assert np.array_equal(acc.view(np.uint32), Ys[b, t].view(np.uint32))
+
+
+# ----------------------------------------------------------------------------- S-normalised metric
+def test_s_normalized_error_and_S_hand_fixture():
+    """s_normalized_error and S = sum |w| (the tolerance denominator of every float
+    assertion) against hand-derived values: cancellation, a 0/0 element (-> 0), a nonzero
+    diff over S = 0 (-> inf), and max over elements (not the mean)."""
+    g = json.load(open(os.path.join(GOLDEN, "s_normalized_error.json")))
+    x = float.fromhex
+    rows = np.array([[x(v) for v in r] for r in g["rows"]], dtype=np.float32)
+    z, S = O.pool_bag_f64(rows)
+    assert np.array_equal(z, np.array([x(v) for v in g["bag_sum"]]))
+    assert np.array_equal(S, np.array([x(v) for v in g["bag_S"]]))
+    offs = np.array(g["table_offsets"], dtype=np.int64)
+    Zt, St = O.pool_table_f64(rows, offs, np.arange(3, dtype=np.int64))
+    assert np.array_equal(Zt, np.array([[x(v) for v in r] for r in g["table_sum"]]))
+    assert np.array_equal(St, np.array([[x(v) for v in r] for r in g["table_S"]]))
+    for c in g["cases"]:
+        y = np.array([x(v) for v in c["y"]])
+        with np.errstate(all="ignore"):
+            got = O.s_normalized_error(y, z, S)
+        if "expected" in c:
+            exp = float("inf") if c["expected"] == "inf" else x(c["expected"])
+        else:
+            exp = x(c["expected_num"]) / x(c["expected_den"])
+        assert got == exp, (c["what"], got, exp)
+
+
+# ----------------------------------------------------------------------------- C7: IEEE specials
+def test_c7_subnormal_sums_not_flushed():
+    """C7 (no FTZ): rows of small multiples of the least subnormal 2^-149 sum exactly
+    (sum_k k * 2^-149 is representable), including sums that stay subnormal and sums
+    that cross into the normal range; a flush-to-zero implementation returns 0."""
+    tiny = np.float32(2.0 ** -149)
+    k = np.array([[1, 3, 7, 2 ** 20], [2, 5, 9, 2 ** 22], [4, 0, 1, 2 ** 23]], dtype=np.int64)
+    W = (k.astype(np.float64) * 2.0 ** -149).astype(np.float32)
+    assert W[0, 0] == tiny and W[2, 3] == np.float32(2.0 ** -126)   # subnormal .. least normal
+    offs = np.array([0, 3, 5], dtype=np.int64)
+    idx = np.array([0, 1, 2, 0, 0], dtype=np.int64)
+    Z = O.pool_table_f32(W, offs, idx)
+    exp = np.array([k.sum(axis=0), 2 * k[0]], dtype=np.float64) * 2.0 ** -149
+    assert np.array_equal(Z.astype(np.float64), exp)
+    assert np.all(Z[:, :3] > 0) and np.all(Z[:, :3] < 2.0 ** -126)     # still subnormal, not flushed
+
+
+def test_c7_inf_nan_propagate_and_negative_zero():
+    """C7 closed forms of IEEE 754 addition: x + Inf = Inf, Inf + (-Inf) = NaN, NaN + x = NaN,
+    overflow of a finite sum -> Inf, (-0) + (-0) = -0 (a bag of -0 rows returns -0, C4)."""
+    big = np.float32(3.0e38)
+    W = np.array([[1.0, np.inf, np.nan, big, -0.0],
+                  [2.0, -np.inf, 1.0, big, -0.0]], dtype=np.float32)
+    offs = np.array([0, 1, 3], dtype=np.int64)
+    with np.errstate(all="ignore"):
+        Z = O.pool_table_f32(W, offs, np.array([0, 0, 1], dtype=np.int64))
+    keep = [0, 1, 3, 4]                                                  # one-hot bag: the row's bits
+    assert np.array_equal(Z[0, keep].view(np.uint32), W[0, keep].view(np.uint32)) and np.isnan(Z[0, 2])
+    assert Z[1, 0] == 3.0 and np.isnan(Z[1, 1]) and np.isnan(Z[1, 2]) and Z[1, 3] == np.inf
+    assert Z[1, 4] == 0 and np.signbit(Z[1, 4])
+
+
+def test_c7_bf16_rounding_of_specials_matches_torch():
+    """rne_bf16 on NaN / +-Inf / subnormals / overflowing finites: NaN stays NaN (the plain
+    rounding rule would turn a low-payload NaN into Inf), everything else bit-equal to
+    torch's float -> bf16 conversion."""
+    torch = pytest.importorskip("torch")
+    u = np.array([0x7F800001, 0xFF800001, 0x7FC00000, 0x7F800000, 0xFF800000, 0x00000001, 0x80000001,
+                  0x00007FFF, 0x00008000, 0x00018000, 0x007FFFFF, 0x7F7FFFFF, 0x7F7F8000, 0xFF7FFFFF,
+                  0x80000000, 0x00000000], dtype=np.uint32)
+    x = u.view(np.float32)
+    got = O.rne_bf16(x)
+    ref = torch.from_numpy(x.copy()).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    nan = np.isnan(x)
+    assert np.all(np.isnan(O.bf16_to_f32(got[nan])))
+    assert np.array_equal(got[~nan], ref[~nan])
+    assert got[3] == 0x7F80 and got[4] == 0xFF80 and got[11] == 0x7F80     # Inf, -Inf, overflow -> Inf
