@@ -273,6 +273,28 @@ def reference_arm(args):
     return 0
 
 
+# ------------------------------------------------------------------------------ roofline over ranks
+def rank_roof(hbm_bytes, egress, ingress, peak, nvl_peak=NVLINK_GBS):
+    """One rank's roofline time (s): the slower of its HBM-compulsory bytes over the HBM peak
+    and its NVLink bytes (max of egress and ingress) over the link bandwidth."""
+    return max(hbm_bytes / (peak * 1e9), max(egress, ingress) / (nvl_peak * 1e9))
+
+
+def combine_roofline(per_rank, ms, peak, nvl_peak=NVLINK_GBS):
+    """frac = max_r t_roof,r / max_r t_measured,r.  per_rank: the all-gathered
+    dicts of every rank; ms: the max-over-ranks measured time per step."""
+    binding = max(per_rank, key=lambda d: d["t_roof_ms"])
+    b_hbm = binding["hbm_compulsory_bytes"] / (peak * 1e9)
+    b_nvl = max(binding["nvlink_egress_bytes"], binding["nvlink_ingress_bytes"]) / (nvl_peak * 1e9)
+    bound = "hbm" if b_hbm >= b_nvl else "nvlink"
+    nbytes = binding["hbm_compulsory_bytes"] if bound == "hbm" else max(binding["nvlink_egress_bytes"],
+                                                                         binding["nvlink_ingress_bytes"])
+    pk = peak if bound == "hbm" else nvl_peak
+    return {"binding": binding, "bound": bound, "bytes": nbytes, "peak": pk,
+            "achieved": nbytes / (ms * 1e-3) / 1e9, "frac": binding["t_roof_ms"] / ms,
+            "t_roof_ms": binding["t_roof_ms"]}
+
+
 # ------------------------------------------------------------------------------ f1 trace summary
 def trace_summary(tr, bins=40):
     """f1 (Figs. 7/10): how the rank's stores spread over its kernel span.
@@ -374,18 +396,24 @@ def combined_clocks(reps, max_mhz):
             "per_repeat_sm_mhz": mhz}
 
 
+def shard_layout(w, S, N):
+    """f3 placement of --shards: table t -> S contiguous row shards, shard s on rank
+    (owner[t] + s) % N; entries (t, s, lo, hi, owner)."""
+    shards = []
+    for t in range(w.T):
+        cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(np.int64)
+        for sh in range(S):
+            shards.append((t, sh, int(cuts[sh]), int(cuts[sh + 1]), (int(w.owner[t]) + sh) % N))
+    return shards
+
+
 def build_shards(args, w, N, rank, H, tables, batches):
     """f3 at any N: table t -> S contiguous row shards, shard s on rank (owner[t] + s) % N.
     Each rank needs the FULL CSR (global row ids) of every table it holds a shard of and the
     rows of its shards; tables are generated (whole) on every rank that holds a shard."""
     import torch
     import synth.gpu as SG
-    S = args.shards
-    shards = []
-    for t in range(w.T):
-        cuts = np.linspace(0, int(w.rows[t]), S + 1).astype(np.int64)
-        for sh in range(S):
-            shards.append((t, sh, int(cuts[sh]), int(cuts[sh + 1]), (int(w.owner[t]) + sh) % N))
+    shards = shard_layout(w, args.shards, N)
     mine = sorted((t, sh, lo, hi) for (t, sh, lo, hi, o) in shards if o == rank)
     need = sorted({t for (t, _, _, _) in mine})
     own_tables = list(w.local_tables(rank))
@@ -556,21 +584,14 @@ def main():
     lookup_bytes = algorithmic_bytes(w, float(np.mean(nnz)), nbags, ib)
     hbm_bytes = float(np.mean([compulsory_bytes(w, u, z, nbags, ib) for u, z in zip(uniq, nnz)]))
     peak, peak_kind = hbm_peak()
-    t_hbm = hbm_bytes / (peak * 1e9)
     t_nvl = max(egress, ingress) / (NVLINK_GBS * 1e9)
-    t_roof_r = max(t_hbm, t_nvl)
+    t_roof_r = rank_roof(hbm_bytes, egress, ingress, peak)
     t_roof = H.allreduce_max(t_roof_r)                    # max_r t_roof,r / max_r t_measured,r
     per_rank = H.gather({"rank": rank, "t_roof_ms": t_roof_r * 1e3, "hbm_compulsory_bytes": hbm_bytes,
                          "lookup_bytes": lookup_bytes, "nvlink_egress_bytes": egress, "nvlink_ingress_bytes": ingress,
                          "unique_rows": float(np.mean(uniq)), "lookups": float(np.mean(nnz))})
-    binding = max(per_rank, key=lambda d: d["t_roof_ms"])
-    b_hbm = binding["hbm_compulsory_bytes"] / (peak * 1e9)
-    b_nvl = max(binding["nvlink_egress_bytes"], binding["nvlink_ingress_bytes"]) / (NVLINK_GBS * 1e9)
-    bound = "hbm" if b_hbm >= b_nvl else "nvlink"
-    bytes_bound = binding["hbm_compulsory_bytes"] if bound == "hbm" else max(binding["nvlink_egress_bytes"],
-                                                                              binding["nvlink_ingress_bytes"])
-    pk = peak if bound == "hbm" else NVLINK_GBS
-    achieved = bytes_bound / (ms * 1e-3) / 1e9
+    rc = combine_roofline(per_rank, ms, peak)
+    binding, bound, bytes_bound, pk, achieved = rc["binding"], rc["bound"], rc["bytes"], rc["peak"], rc["achieved"]
     default_kernel = not args.opt and args.shards == 1 and ib == 8
     traffic, traffic_src, l2 = None, None, None
     if default_kernel:                                    # the committed ncu capture is of the default kernel

@@ -182,7 +182,7 @@ static int fwd_mode(bool check, bool shard, bool tmast) {
 }
 // dynamic shared memory: the per-warp id ring (+ f4: two staging buffers of 4 output rows per warp)
 static size_t fwd_smem(const emb_ctx* c, int mode) {
-  size_t s = (size_t)(kBlock / 32) * kSidxWarpBytes;
+  size_t s = (size_t)(kBlock / 32) * kSidxWarpBytes + kSidxWarpBytes;   // + alignment slack of the rings
   if (mode == kModeTma) s += (size_t)(kBlock / 32) * 8 * (size_t)c->d * esize(c->odt);
   return mode == kModeFilt ? 0 : s;
 }

@@ -80,14 +80,17 @@ class PgasEmbedding:
         return self._send, self._recv, self._out
 
     def forward_baseline(self, offsets: torch.Tensor, indices: torch.Tensor, group=None, flags: int = 0,
-                         stream=None, single_float: bool = False, pool_only: bool = False) -> torch.Tensor:
+                         stream=None, single_float: bool = False, pool_only: bool = False,
+                         always_exchange: bool = False) -> torch.Tensor:
         """pool kernel -> all_to_all_single(async_op=True).wait() -> unpack kernel (L155, L193).
         single_float: the exchange sends ONE float per peer instead of the pooled vectors and the
         unpack still runs over the (stale) receive buffer -- the paper's probe for the
-        sync + unpack share of the exchange phase (L286-292); pool_only: stop after the pool."""
+        sync + unpack share of the exchange phase (L286-292); pool_only: stop after the pool;
+        always_exchange: run the collective + unpack even at G = 1 (a self-exchange)."""
         send, recv, out = self._baseline_buffers()
         E.emb_baseline_pool(self.ctx, offsets, indices, send, flags, stream)
-        if self.ctx.world_size == 1 or pool_only:  # G = 1: send already is [B][T][d]; no exchange, no unpack
+        if (self.ctx.world_size == 1 and not always_exchange) or pool_only:
+            # G = 1: send already is [B][T][d]; no exchange, no unpack
             return send[: self.B_r * self.T * self.dim].view(self.B_r, self.T, self.dim)
         import torch.distributed as dist
         G = self.ctx.world_size

@@ -164,6 +164,30 @@ def test_simulated_ranks_bitexact(G, flags):
         _close(layers)
 
 
+@pytest.mark.parametrize("G,wdt,i32", [(4, "f32", False), (8, "f32", True), (3, "bf16", False)])
+def test_simulated_ranks_medium_size_bitexact(G, wdt, i32):
+    """Multi-rank parity beyond tiny shapes: G ranks (up to the 8 of the scaling run) with
+    16-32 tables of 40 K rows, d = 128, 2-4 K samples and pooling up to 128, LPT-like mixed
+    placement, zipf ids: every element bit-exact (remote stores, chunks crossing rank
+    boundaries of the mini-batch, destination-staggered order)."""
+    T = 4 * G
+    rng = np.random.default_rng(G)
+    owner = rng.permutation(np.arange(T) % G)
+    w = synth.make_workload("tiny", G=G, pmin=1, pmax=128, B=512 * G + 3, T=T, dim=128, rows=40000, dist="zipf",
+                            wdtype=wdt, odtype=wdt, owner=owner)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 61)
+    ref = H.oracle_outputs(w, 61, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, csr, i32=i32)
+        for r in range(G):
+            _assert_exact(got[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)
+
+
 def test_placement_invariance_and_rank_without_tables():
     outs = []
     for own in ([0, 0, 1, 1, 2, 2], [2, 1, 0, 2, 1, 0], [1, 1, 1, 1, 1, 1], [0, 2, 0, 2, 0, 2]):
@@ -179,14 +203,14 @@ def test_placement_invariance_and_rank_without_tables():
 
 
 def test_epoch_ring_poisoned_slots_exactly_once():
-    """P14: every returned slot is poisoned with NaN after it is read; the 2-slot ring
-    rewrites it two epochs later, so from epoch 2 on every forward lands on poison and
+    """P14: every returned slot is poisoned with NaN after it is read; the 3-slot ring
+    rewrites it three epochs later, so from epoch 3 on every forward lands on poison and
     must leave no NaN and match the oracle (exactly-once, C21)."""
     w = synth.make_workload("tiny", G=2, pmin=0, pmax=12, B=90, T=5, dim=32, rows=300)
     tabs = H.np_tables(w)
     layers = _layers(w, tabs)
     try:
-        for epoch in range(6):
+        for epoch in range(8):
             csr = H.np_csrs(w, 1000 + epoch)
             ref = H.oracle_outputs(w, 1000 + epoch, tabs, csr)
             offs, idxs = csr

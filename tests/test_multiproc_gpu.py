@@ -233,3 +233,59 @@ def test_cross_process_ipc_backward(G):
         assert tb == "", tb
         assert ok, f"rank {rank} dW != oracle"
         assert err == 0, f"rank {rank} device error {err}"
+
+
+def _nccl_worker(port, q):
+    """The comparison path's NCCL branch (layer.forward_baseline: all_to_all_single with
+    async_op=True + wait, then the unpack kernel) on a real NCCL process group.  NCCL refuses
+    two ranks on one GPU ("Duplicate GPU detected", tools/probe_nccl_same_gpu.py), so this
+    runs world size 1 and forces the exchange (a self all-to-all)."""
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    try:
+        import torch.distributed as dist
+
+        import emb_test_helpers as H
+        import synth
+        from paper_conf_sc_chenbyo24_b200.layer import PgasEmbedding
+
+        torch.cuda.set_device(0)
+        dev = torch.device("cuda", 0)
+        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1, device_id=dev)
+        assert dist.get_backend() == "nccl"
+        w = synth.make_workload("tiny", G=1, pmin=0, pmax=25, B=97, T=6, dim=64, rows=600)
+        tabs = H.np_tables(w)
+        layer = PgasEmbedding(0, 1, 0, w.rows, w.owner, w.dim, [torch.from_numpy(tabs[t]).to(dev) for t in range(w.T)],
+                              w.B)
+        o, x = synth.rank_csr(w, 321, 0)
+        od, xd = torch.from_numpy(o).to(dev), torch.from_numpy(x).to(dev)
+        ref = H.oracle_outputs(w, 321, tabs)[0]
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            y = layer.forward_baseline(od, xd, None, 0, s, always_exchange=True)
+        s.synchronize()
+        ok = np.array_equal(y.cpu().numpy().view(np.uint32), ref.view(np.uint32))
+        with torch.cuda.stream(s):                  # the paper's one-float probe runs too
+            layer.forward_baseline(od, xd, None, 0, s, single_float=True, always_exchange=True)
+        s.synchronize()
+        err = layer.device_error()
+        layer.close()
+        dist.destroy_process_group()
+        q.put((0, bool(ok), int(err), ""))
+    except Exception:
+        import traceback
+        q.put((0, False, -1, traceback.format_exc()))
+
+
+def test_nccl_comparison_path_executes():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_worker, args=(_port(), q))
+    p.start()
+    rank, ok, err, tb = q.get(timeout=300)
+    p.join(timeout=60)
+    assert tb == "", tb
+    assert ok, "NCCL comparison path output != oracle"
+    assert err == 0

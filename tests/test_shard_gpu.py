@@ -99,3 +99,83 @@ def test_sharded_all_shards_on_one_rank_and_rank_without_shards():
     w = synth.make_workload("tiny", G=3, pmin=0, pmax=25, B=50, T=3, dim=128, rows=500)
     shards = _shards(w, lambda t: 3, lambda t, s: 1)  # everything on rank 1, ranks 0/2 only consume
     _run(w, shards, [7])
+
+
+def _run_plain(w, shards, seed, flags=0, bad=None):
+    """Sharded forward on the GPU; returns (outputs, device errors, offs, idxs)."""
+    tabs = H.np_tables(w)
+    full = [tabs[int(w.phys[t])] for t in range(w.T)]
+    dev_full = [torch.from_numpy(a).to(DEV) for a in full]
+    local_w = [[dev_full[t][lo:hi] for (t, s, lo, hi, o) in sorted(shards) if o == r] for r in range(w.G)]
+    grp = LocalGroup(w.G) if w.G > 1 else None
+    layers = run_ranks(w.G, lambda r: PgasEmbedding(r, w.G, 0, w.rows, None, w.dim, local_w[r], w.B, w.wdtype,
+                                                    w.odtype, grp.allgather_for(r) if grp else None,
+                                                    {"timeout_ms": 20000}, shards=shards))
+    try:
+        offs, idxs = _inputs(w, seed, shards)
+        if bad is not None:
+            idxs = [bad(r, x.copy()) for r, x in enumerate(idxs)]
+        ins = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(w.G)]
+        streams = [torch.cuda.Stream() for _ in range(w.G)]
+        torch.cuda.synchronize()
+        ys = [layers[r].forward(ins[r][0], ins[r][1], flags, streams[r]) for r in range(w.G)]
+        torch.cuda.synchronize()
+        got = [H.dev_out_to_np(y.clone()) for y in ys]
+        errs = [layers[r].device_error(clear=True) for r in range(w.G)]
+    finally:
+        run_ranks(w.G, lambda r: layers[r].close())
+    return got, errs, full
+
+
+@pytest.mark.parametrize("G", [1, 2, 3])
+def test_sharded_equals_plain_unsharded_definition(G):
+    """f3 against the PLAIN definition of the forward (no shards: Y_r[i, t] = sum over the
+    bag in CSR order, O.emb_forward with a table-wise placement), not the sharded oracle:
+    integer-valued tables make every summation order exact, so the sharded GPU output must
+    equal it bit for bit; float tables stay within the north star's 1e-6 S-normalised bound."""
+    for mode in ("int", "float"):
+        w = synth.make_workload("tiny", G=G, pmin=0, pmax=60, B=67, T=4, dim=32, rows=800, dist="zipf", mode=mode)
+        shards = _shards(w, lambda t: [3, 1, 2, 4][t], lambda t, s: (t + s) % G)
+        got, errs, full = _run_plain(w, shards, 41)
+        assert errs == [0] * G
+        wt = synth.make_workload("tiny", G=1, pmin=0, pmax=60, B=67, T=4, dim=32, rows=800, dist="zipf", mode=mode)
+        o1, x1 = synth.rank_csr(wt, 41, 0)                # table-wise, one rank: the plain definition
+        plain = O.emb_forward(full, wt.owner, [o1], [x1], w.B, 1)[0]
+        cat = np.concatenate(got, axis=0)
+        if mode == "int":
+            assert np.array_equal(cat.view(np.uint32), plain.view(np.uint32))
+        else:
+            for t in range(w.T):
+                lo, hi = O.rank_table_csr(o1, t, w.B)[1:]
+                z64, S = O.pool_table_f64(full[t], O.rank_table_csr(o1, t, w.B)[0], x1[lo:hi])
+                assert O.s_normalized_error(cat[:, t], z64, S) <= 1e-6
+
+
+def test_sharded_check_bounds():
+    """EMB_FWD_CHECK_BOUNDS with row-sharded tables: ids outside the whole table's [0, M_t)
+    are flagged on the rank that scans them and contribute nothing; ids of another shard
+    are skipped silently."""
+    G = 2
+    w = synth.make_workload("tiny", G=G, pmin=1, pmax=20, B=40, T=2, dim=32, rows=300, mode="int")
+    shards = _shards(w, lambda t: 2, lambda t, s: s)
+
+    def bad(r, x):
+        x[2] = 300 if r == 0 else -1
+        return x
+    got, errs, full = _run_plain(w, shards, 9, E.EMB_FWD_CHECK_BOUNDS, bad=bad)
+    assert all(e & E.EMB_DEVERR_BOUNDS for e in errs)
+    # expected: the plain definition over the ids that are in range (integer tables: exact)
+    offs, idxs = _inputs(w, 9, shards)
+    idxs = [bad(r, x.copy()) for r, x in enumerate(idxs)]
+    exp = np.zeros((w.B, w.T, w.dim), np.float32)
+    for r in range(G):                                    # rank r holds shard r of every table
+        for k, t in enumerate(range(w.T)):
+            o, lo, hi = O.rank_table_csr(offs[r], k, w.B)
+            for b in range(w.B):
+                xs = [int(v) for v in idxs[r][lo + o[b]: lo + o[b + 1]]]
+                lo_r, hi_r = [(s_lo, s_hi) for (tt, s, s_lo, s_hi, own) in shards if tt == t and own == r][0]
+                for v in xs:
+                    if lo_r <= v < hi_r:
+                        exp[b, t] += full[t][v]
+    cat = np.concatenate(got, axis=0)
+    assert np.array_equal(cat, exp)
