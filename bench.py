@@ -10,8 +10,9 @@ One JSON line on rank 0.  A "step" is one whole EMB forward (lookup + pool + MP-
 exchange, PAPER.md L197 timed scope) over one batch of synthetic Criteo-shaped input
 already resident in HBM.  Every timed figure is the median of `--repeats` (5) runs of K
 steps, each bracketed by a barrier + synchronize, device-timed with CUDA events on the
-launching stream and max-reduced over ranks (SURVEY §8(d) timing protocol); the clocks of
-every repeat are recorded.  `e2e` repeats it through the public C ABI with pinned host CSR
+launching stream and max-reduced over ranks (SURVEY §8(d) timing protocol); every repeat
+starts after `--repeat-gap` (1 s) idle so it does not inherit the previous repeat's power
+capping, and the clocks of every repeat are recorded.  `e2e` repeats it through the public C ABI with pinned host CSR
 in and the host output out.  `--impl reference` times the CPU oracle (this tier's reference
 arm) on a bounded sample of the same workload.  Nothing here reads /root/reference.
 """
@@ -42,6 +43,9 @@ def parse():
     p.add_argument("--steps", type=int, default=100)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--repeats", type=int, default=5, help="timed repeats of K steps; the median is reported")
+    p.add_argument("--repeat-gap", type=float, default=1.0,
+                   help="idle seconds before every repeat (the power controller recovers, so a repeat does not "
+                        "inherit the previous one's sw_power_cap clock; per-repeat clocks are recorded)")
     p.add_argument("--config", default="weak")
     p.add_argument("--dist", default=None, help="override index distribution (zipf|uniform)")
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -382,6 +386,13 @@ class Harness:
         """median over `repeats` device-timed runs of `steps` steps (max over ranks each)"""
         reps = []
         for _ in range(max(self.args.repeats, 1)):
+            if self.args.repeat_gap > 0:
+                self.torch.cuda.synchronize()
+                time.sleep(self.args.repeat_gap)
+                for s in range(2):                        # clocks back up from idle (untimed)
+                    fn(s)
+                if finish is not None:
+                    finish()
             with ClockSampler(self.local) as clk:
                 ms = self.timed_once(fn, steps, finish)
             reps.append({"ms": ms, **{k: v for k, v in clk.summary().items() if k in ("sm_mhz", "reasons")}})
@@ -756,8 +767,8 @@ def main():
         H.dist.barrier()
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N,
-                "steps": args.steps, "warmup": args.warmup, "repeats": len(reps), "ms_per_step": ms,
-                "ms_per_step_repeats": [r["ms"] for r in reps], "higher_is_better": True,
+                "steps": args.steps, "warmup": args.warmup, "repeats": len(reps), "repeat_gap_s": args.repeat_gap,
+                "ms_per_step": ms, "ms_per_step_repeats": [r["ms"] for r in reps], "higher_is_better": True,
                 "scaling": "weak" if w.name.startswith("weak") else "strong", "vs_baseline": None,
                 "dtype": "f32" if (w.wdtype == "f32") else "bf16", "data": "synthetic",
                 "config": config_desc(w, N, args), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
