@@ -603,13 +603,14 @@ def main():
                          "unique_rows": float(np.mean(uniq)), "lookups": float(np.mean(nnz))})
     rc = combine_roofline(per_rank, ms, peak)
     binding, bound, bytes_bound, pk, achieved = rc["binding"], rc["bound"], rc["bytes"], rc["peak"], rc["achieved"]
-    default_kernel = not args.opt and args.shards == 1 and ib == 8
+    default_kernel = not args.opt and args.shards == 1
     traffic, traffic_src, l2 = None, None, None
     if default_kernel:                                    # the committed ncu capture is of the default kernel
         try:
             with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
                 tj = json.load(f)
-            key = f"{w.name}:{w.dist}:G{N}"  # profiles/traffic.json: ncu --set full of this workload
+            # profiles/traffic.json: ncu --set full of this workload (":i32": the int32-index run)
+            key = f"{w.name}:{w.dist}:G{N}" + (":i32" if ib == 4 else "")
             if key in tj:
                 traffic = tj[key]["dram_bytes_per_launch"]
                 traffic_src = tj[key].get("source")

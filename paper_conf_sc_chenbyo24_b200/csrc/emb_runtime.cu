@@ -119,8 +119,8 @@ struct emb_ctx {
   size_t p_offcap[2] = {0, 0};            // bytes of p_off[k]
   cudaStream_t s_in = nullptr, s_out = nullptr;
   cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr};
-  cudaEvent_t ev_out[kOutSlots] = {nullptr, nullptr, nullptr};   // D2H of the output of epoch e, by e % kOutSlots
-  bool kern_rec[2] = {false, false}, out_rec[kOutSlots] = {false, false, false};
+  cudaEvent_t ev_out[kOutSlots] = {};   // D2H of the output of epoch e, by e % kOutSlots
+  bool kern_rec[2] = {false, false}, out_rec[kOutSlots] = {};
   uint64_t host_calls = 0;
   bool wait_pending = false;            // last forward used EMB_FWD_SEPARATE_WAIT and emb_wait is due
   // f2 backward

@@ -82,6 +82,6 @@ def test_bench_int32_and_shards_lines():
                            timeout=600)
         assert r.returncode == 0, r.stderr[-3000:]
         d = _last_json(r.stdout)
-        assert d["value"] > 0 and d["roofline"]["traffic"] is None
+        assert d["value"] > 0 and (d["roofline"]["traffic"] is None or extra[0] == "--index-bits")
         if extra[0] == "--index-bits":
             assert d["config"]["index_bits"] == 32 and "i32" in d["e2e"]["path"]

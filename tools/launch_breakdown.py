@@ -1,12 +1,23 @@
-import csv, sys
+"""Per-kernel share of an ncu launch list (ncu --metrics gpu__time_duration.sum ... --csv):
+cold-cache, serialised times, so compare SHARES, not absolutes."""
+import collections
+import csv
+import sys
+
 for f in sys.argv[1:]:
-    rows=[r for r in csv.reader(open(f)) if r and (r[0]=="ID" or r[0].isdigit())]
-    h=rows[0]; ik=h.index("Kernel Name"); im=h.index("Metric Name"); iv=h.index("Metric Value"); ii=h.index("ID")
-    agg={}
+    rows = [r for r in csv.reader(open(f)) if r and (r[0] == "ID" or r[0].isdigit())]
+    h = rows[0]
+    ik, im, iv, iu = h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Value"), h.index("Metric Unit")
+    tot = collections.defaultdict(float)
+    n = collections.Counter()
     for r in rows[1:]:
-        agg.setdefault((r[ii],r[ik][:40]),{})[r[im]]=r[iv]
-    print(f); tot=0
-    for (i,k),m in list(agg.items())[-6:]:
-        t=float(m['gpu__time_duration.sum'].replace(',',''))/1e3; tot+=t
-        print(f"  {k:40s} {t:8.1f} us  rd {float(m['dram__bytes_read.sum'].replace(',',''))/1e9:6.2f} GB wr {float(m['dram__bytes_write.sum'].replace(',',''))/1e9:6.2f} GB")
-    print("  total", round(tot,1))
+        if r[im] != "gpu__time_duration.sum":
+            continue
+        scale = {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}.get(r[iu], 1e-3)
+        k = r[ik].split("(")[0][:60]
+        tot[k] += float(r[iv].replace(",", "")) * scale
+        n[k] += 1
+    s = sum(tot.values()) or 1.0
+    print(f)
+    for k, t in sorted(tot.items(), key=lambda kv: -kv[1]):
+        print(f"  {k:60s} launches {n[k]:4d}  {t / n[k]:9.1f} us/launch  share {100 * t / s:5.1f} %")
