@@ -320,12 +320,14 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
   }
   // completion: every CTA's reads of peer slots are done before the last CTA tells the
   // peers their slots may be refilled
+  // (G = 1: no peer waits for "done", so device scope suffices, as in cta_complete)
   __syncthreads();
   if (threadIdx.x != 0) return;
-  fence_acq_rel_sys();
+  if (p.G > 1) fence_acq_rel_sys();
   const unsigned prev = atomicAdd(&p.ctrl->bdone, 1u);
   if (prev != gridDim.x - 1) return;
-  fence_acq_rel_sys();
+  if (p.G > 1) fence_acq_rel_sys();
+  else __threadfence();
   p.ctrl->bdone = 0;
   p.ctrl->bwork = 0;
   for (int q = 1; q < p.G; ++q) st_release_sys(p.peer_done[(p.rank + q) % p.G], p.epoch);
