@@ -471,8 +471,8 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     }
     cudaFuncGetAttributes(&a, emb_wait_kernel);
     cudaFuncGetAttributes(&a, emb_sleep_kernel);
-    cudaFuncGetAttributes(&a, emb_unpack_kernel);
-    cudaFuncGetAttributes(&a, emb_unpack8_kernel);
+    cudaFuncGetAttributes(&a, emb_unpack_rows_kernel<uint4>);
+    cudaFuncGetAttributes(&a, emb_unpack_rows_kernel<uint2>);
     cudaFuncGetAttributes(&a, emb_combine_kernel<float>);
     cudaFuncGetAttributes(&a, emb_combine_kernel<__nv_bfloat16>);
     cudaFuncGetAttributes(&a, emb_bwd_signal_kernel);
@@ -1293,15 +1293,17 @@ emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, v
   CK(c, cudaSetDevice(c->dev));
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
   const int rowbytes = c->d * (int)esize(c->odt);
-  const int64_t pieces = Br * c->T * (rowbytes % 16 == 0 ? rowbytes / 16 : rowbytes / 8);
-  int grid = (int)std::min<int64_t>((pieces + kBlock - 1) / kBlock, (int64_t)c->num_sms * 8);
+  const int64_t rows = Br * c->T;
+  int grid = (int)std::min<int64_t>((rows + (kBlock / 32) - 1) / (kBlock / 32), (int64_t)c->num_sms * 8);
   if (grid < 1) grid = 1;
   if (rowbytes % 16 == 0)
-    emb_unpack_kernel<<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out, c->d_unpack_base,
-                                                                  c->d_unpack_stride, Br, c->T, rowbytes);
+    emb_unpack_rows_kernel<uint4><<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out,
+                                                                           c->d_unpack_base, c->d_unpack_stride, Br,
+                                                                           c->T, rowbytes);
   else
-    emb_unpack8_kernel<<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out, c->d_unpack_base,
-                                                                   c->d_unpack_stride, Br, c->T, rowbytes);
+    emb_unpack_rows_kernel<uint2><<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out,
+                                                                           c->d_unpack_base, c->d_unpack_stride, Br,
+                                                                           c->T, rowbytes);
   CK(c, cudaGetLastError());
   return EMB_OK;
 }

@@ -164,6 +164,27 @@ def test_simulated_ranks_bitexact(G, flags):
         _close(layers)
 
 
+def test_simulated_ranks_max_world_size():
+    """kMaxG = 16 simulated ranks (the largest world size the kernel parameters carry):
+    every rank owns one or two tables, uneven mini-batches (B mod G != 0), remote stores to
+    15 peers, flags from 15 sources; bit-exact; a 17th rank is refused."""
+    G = 16
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=9, B=16 * 7 + 5, T=24, dim=32, rows=200)
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 23)
+    ref = H.oracle_outputs(w, 23, tabs, csr)
+    layers = _layers(w, tabs)
+    try:
+        got = _run(w, layers, csr)
+        for r in range(G):
+            _assert_exact(got[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)
+    with pytest.raises(E.EmbError):
+        E.emb_init(0, 17, 0, lambda b: b * 17)
+
+
 @pytest.mark.parametrize("G,wdt,i32", [(4, "f32", False), (8, "f32", True), (3, "bf16", False)])
 def test_simulated_ranks_medium_size_bitexact(G, wdt, i32):
     """Multi-rank parity beyond tiny shapes: G ranks (up to the 8 of the scaling run) with
