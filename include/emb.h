@@ -159,8 +159,8 @@ emb_status_t emb_register_sharded_tables(emb_ctx_t* ctx, int32_t num_tables, con
  * Without EMB_FWD_SEPARATE_WAIT the kernel completes only when every peer's
  * pooled vectors for this rank have landed (in-kernel acquire wait), so any later
  * work on `stream` sees the whole Y_r.  With it, emb_wait completes the forward; a
- * forward issued while the previous one's emb_wait is still due enqueues that wait
- * first.  Empty bags produce +0.0 (C2).  IEEE fp32 adds, no flush-to-zero; NaN and
+ * forward issued while the previous one's emb_wait is still due enqueues that wait on its
+ * own `stream` first (if the two forwards use different streams, the caller orders them).  Empty bags produce +0.0 (C2).  IEEE fp32 adds, no flush-to-zero; NaN and
  * Inf propagate (C7).  Unknown flag bits: EMB_ERR_ARG.
  * Errors: EMB_ERR_STATE (not registered), EMB_ERR_ARG, EMB_ERR_CUDA.  Device-side
  * failures (peer timeout, bounds) set the sticky device error word instead. */
