@@ -53,7 +53,10 @@ def parse():
                    help="backward = SURVEY row f2 (emb_backward: pull output gradients, scatter into dW)")
     p.add_argument("--index-bits", type=int, default=64, choices=[64, 32],
                    help="CSR index/offset width (C12: int64 is the paper's; int32 halves the index bytes)")
-    p.add_argument("--batches", type=int, default=4, help="distinct pre-generated batches cycled")
+    p.add_argument("--batches", type=int, default=None,
+                   help="distinct pre-generated batches cycled (default 4; 2 for `large`, whose 150 GB of tables "
+                        "per rank leave room for two 1.7 GB index batches next to the output ring and the "
+                        "comparison buffers, SURVEY §8(d))")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-control", action="store_true", help="skip the uniform-index control measurement")
@@ -541,6 +544,8 @@ def main():
     H = Harness(args)
     N, rank, dev, stream = H.N, H.rank, H.dev, H.stream
     w = synth.make_workload(args.config, G=N, dist=args.dist)
+    if args.batches is None:
+        args.batches = 2 if args.config == "large" else 4
     ib = args.index_bits // 8
 
     # ---- inputs in HBM (untimed)

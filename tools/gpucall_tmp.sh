@@ -1,6 +1,5 @@
 set -u
-O=gpurun_out/r02p; mkdir -p $O
-timeout 1800 python -m pytest tests -m gpu -x -q > $O/tests.log 2>&1; tail -n 1 $O/tests.log
-for L in exp_so/libemb_cur.so exp_so/libemb_unpack2.so exp_so/libemb_cur.so exp_so/libemb_unpack2.so; do
-  echo "$L $(EMB_LIB=$L python tools/unpack_probe.py 2>&1 | tail -1)"
-done | tee $O/unpack.txt
+O=gpurun_out/r02r; mkdir -p $O
+python tools/sweep.py --config weak --dists zipf,uniform --steps 100 --gap 2 --repeat 4 --opts "" "tail_div=8" "tail_div=16" "tail_div=8,chunk_rows=160" 2>&1 | tee $O/sweep_weak.txt | grep summary
+python tools/sweep.py --config single --dists zipf --steps 100 --gap 2 --repeat 4 --opts "" "tail_div=8" "tail_div=16" 2>&1 | tee $O/sweep_single.txt | grep summary
+python tools/sweep.py --config large_shard --dists zipf --steps 30 --gap 2 --repeat 2 --opts "" "tail_div=8" 2>&1 | tee $O/sweep_ls.txt | grep summary

@@ -32,6 +32,8 @@ for spec in "weak_zipf:" "weak_uniform:--dist uniform" "single_zipf:--config sin
 done
 ncu --set full --clock-control none --import-source on -k regex:emb_bwd_kernel -s 3 -c 1 -o $O/full_weak_zipf_backward -f \
     $NB --mode backward > $O/full_bwd.log 2>&1
+python tools/pcie_bw.py > $O/pcie_bw.txt 2>&1
+python tools/unpack_probe.py > $O/unpack_probe.txt 2>&1
 for t in memcheck racecheck synccheck; do
   compute-sanitizer --tool $t --kernel-name kns=emb python tools/sanitize.py > $O/san_$t.log 2>&1
 done
