@@ -3,7 +3,7 @@
 # the default bench command, full ncu captures of the hot kernels, compute-sanitizer.
 # Output under gpurun_out/r02m/ (summaries are copied to profiles/r02/ afterwards).
 set -u
-O=gpurun_out/r02m; mkdir -p $O
+O=${OUT:-gpurun_out/r02m}; mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv > $O/smi.txt 2>&1
 B="python bench.py"
 $B > $O/bench_r02.json 2> $O/bench_r02.err
