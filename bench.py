@@ -563,8 +563,7 @@ def main():
     if args.shards > 1:
         if args.mode == "backward":
             raise SystemExit("--shards > 1 has no backward (f2 is table-wise)")
-        args.no_control = True       # the uniform control and the comparison path are table-wise
-        args.no_compare = True
+        args.no_control = True       # the uniform control is table-wise
         shards, tables, batches, stat_tables, ranges = build_shards(args, w, N, rank, H, tables, batches)
         torch.cuda.synchronize()
     nnz = [int(b[0][-1].item()) for b in batches]
@@ -698,7 +697,8 @@ def main():
         ms_b, _ = H.timed(run_b(False), k_b, what="nccl_path")
         cmp = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3), "pgas_speedup": ms_b / ms}
         if N == 1:
-            cmp["note"] = "G=1: pool kernel only (no exchange, no unpack)"
+            cmp["note"] = ("G=1: pool kernel + the partials' combine (no exchange)" if shards is not None else
+                           "G=1: pool kernel only (no exchange, no unpack)")
             cmp["breakdown"] = {"computation_ms": ms_b, "communication_ms": 0.0, "sync_unpack_ms": 0.0}
         else:
             for s in range(3):

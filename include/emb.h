@@ -138,8 +138,13 @@ emb_status_t emb_register_tables(emb_ctx_t* ctx, int32_t num_tables, const int64
  * other shards' ids (in-kernel partitioning), stores each bag's fp32 partial sum into the
  * owner's partial slot (one-sided, like the pooled vectors), and after the exchange a
  * combine kernel sums the partials in shard order into Y_r (bf16 out: RNE once).
- * EMB_FWD_CHECK_BOUNDS checks ids against the whole table's [0, rows[t]).  Not supported
- * with row-sharded tables: the comparison path, backward.  Errors as emb_register_tables. */
+ * EMB_FWD_CHECK_BOUNDS checks ids against the whole table's [0, rows[t]).  Backward (f2,
+ * bwd_algo 0): the same CSR; each shard owner accumulates into its shard's rows only (dW of a
+ * local shard is [hi - lo][d], shard-local rows).  Comparison path: emb_baseline_pool writes
+ * every local shard's fp32 partial (whole tables too) destination-major, the splits count fp32
+ * elements, and emb_baseline_unpack sums each table's partials in shard order (then RNE for
+ * bf16 out) -- the same result as the fused path, bit for bit.  Not supported with row-sharded
+ * tables: bwd_algo 1.  Errors as emb_register_tables. */
 emb_status_t emb_register_sharded_tables(emb_ctx_t* ctx, int32_t num_tables, const int64_t* rows,
                                          const int32_t* num_shards, const int32_t* shard_owner,
                                          const int64_t* shard_row_start, int32_t dim, emb_dtype_t weight_dtype,
@@ -280,8 +285,9 @@ emb_status_t emb_query_device_error(emb_ctx_t* ctx, uint32_t* word, int clear);
 const char* emb_last_error(const emb_ctx_t* ctx);
 
 /* ---- comparison path (L155, L193) -------------------------------
- * Split sizes (in ELEMENTS of out dtype) for torch.distributed.all_to_all_single:
- * send_counts[dst] = B_dst*T_r*d, recv_counts[src] = B_r*T_src*d. */
+ * Split sizes (in ELEMENTS of out dtype; fp32 elements with row-sharded tables) for
+ * torch.distributed.all_to_all_single: send_counts[dst] = B_dst*T_r*d,
+ * recv_counts[src] = B_r*T_src*d (T_r, T_src: local tables or, sharded, local shards). */
 emb_status_t emb_baseline_splits(const emb_ctx_t* ctx, int64_t* send_counts, int64_t* recv_counts);
 
 /* Same gather+pool core as emb_forward, written destination-major into the

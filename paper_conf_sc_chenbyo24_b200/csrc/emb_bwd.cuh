@@ -6,7 +6,8 @@
 // direct-GPU remote [accesses]".  Definition (adjoint of sum pooling, L91-95):
 //     dW_t[x, :] = sum over bags (t, b), positions j with x_t[j] = x, of dY[b, t, :]
 // where dY[b] lives on the rank owning sample b (data parallel) and dW_t on the owner of
-// table t (model parallel).
+// table t (model parallel) -- or, for an f3 row-sharded table, the rows [lo, hi) of dW_t on
+// the shard's owner, which reads the table's full bag list and keeps its own ids.
 //
 // B200 design: the OWNER pulls.  Every rank writes its dY [B_r][T][d] (fp32) into a
 // symmetric grad slot and releases a per-source "ready" flag; the owner's fused kernel
@@ -152,7 +153,12 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
       const int64_t o_l = (lane <= nb) ? ld_stream_i64(p.offsets + (int64_t)t_l * B + b0 + lane) : 0;
       const TableDesc* tdp = p.tables + t_l;
       const int64_t tglob = __ldg(&tdp->tglob);
-      const bool pack = __ldg(reinterpret_cast<const long long*>(&tdp->rows)) < (1ll << 26);
+      const int64_t trows = __ldg(reinterpret_cast<const long long*>(&tdp->rows));
+      const bool pack = trows < (1ll << 26);
+      // f3 row shards: the CSR lists the table's full bags with global row ids; ids outside
+      // this shard's [lo, lo + rows) belong to another shard's owner and are skipped (a whole
+      // table has lo = 0, rows = M_t: nothing is skipped)
+      const uint32_t tlo = (uint32_t)__ldg(reinterpret_cast<const long long*>(&tdp->lo));
       char* dwl = reinterpret_cast<char*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t_l))) + lane * VB;
 
       auto gaddr = [&](int bag) -> const char* {        // dY[b][tglob] on the DP rank owning b
@@ -211,8 +217,12 @@ __global__ void __launch_bounds__(kBlock) emb_bwd_kernel(const __grid_constant__
           }
           __syncwarp();
           uint32_t x = 0x80000000u | lane;
-          if (c0 + lane < e0)
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(ring_s + (uint32_t)(((r0 + lane) & 127) * 4)) : "memory");
+          if (c0 + lane < e0) {
+            uint32_t xg;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(xg) : "r"(ring_s + (uint32_t)(((r0 + lane) & 127) * 4)) : "memory");
+            const uint32_t xs = xg - tlo;                 // shard-local row
+            if ((uint64_t)xs < (uint64_t)trows) x = xs;
+          }
           const unsigned same = __match_any_sync(kFull, x);
           const bool lead = (x & 0x80000000u) == 0 && (__ffs(same) - 1) == lane;
           const unsigned leaders = __ballot_sync(kFull, lead);

@@ -90,6 +90,10 @@ struct emb_ctx {
   std::vector<uint64_t> peer_part_off, peer_pslot_bytes;
   int32_t* d_comb_tglob = nullptr;
   int32_t* d_comb_nsh = nullptr;
+  int64_t* d_pbase = nullptr;           // f3 comparison path: unpack-combine maps
+  int32_t* d_pstride = nullptr;
+  int32_t* d_psoff = nullptr;
+  std::vector<int32_t> nloc;            // f3: local shards (incl. whole tables) of every rank
   std::vector<int32_t> tables_of[kMaxG];
   TableDesc* d_tables = nullptr;
   // symmetric buffer (flags at offset 0, slots after)
@@ -287,6 +291,7 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
   struct LocalShard { int t, s, part; int64_t lo, hi; };
   std::vector<LocalShard> lsh;
   std::vector<int32_t> comb_tglob, comb_nsh;
+  std::vector<int32_t> ent_owner, ent_k, ent_off(1, 0), nloc(c->G, 0);   // every (t, s): owner, its index there
   c->T_sh = 0;
   c->S_max = 1;
   for (int t = 0; t < num_tables; ++t)
@@ -313,12 +318,15 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
         c->owner[t] = o;
         c->tables_of[o].push_back(t);
       }
+      ent_owner.push_back(o);
+      ent_k.push_back(nloc[o]++);
       if (o == c->rank) {
         lsh.push_back({t, sh, S > 1 ? ksh * c->S_max + sh : -1, lo, hi});
         c->local.push_back(t);
       }
     }
     if (S > 1) ++ksh;
+    ent_off.push_back((int32_t)ent_owner.size());
   }
   c->has_shard = c->T_sh > 0;
   c->T_r = (int)c->local.size();
@@ -343,6 +351,23 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     td[i].lo = lsh[i].lo;
   }
   if (c->has_shard) {
+    // f3 comparison path: recv = [G][B_r][T_loc(src)][d] fp32 partials; the partial of shard
+    // (t, s) for sample b is vector R0[src] + b * T_loc(src) + k (k = its index on src)
+    const int64_t Br0 = c->bstart[c->rank + 1] - c->bstart[c->rank];
+    std::vector<int64_t> R0(c->G + 1, 0), pbase(ent_owner.size());
+    std::vector<int32_t> pstride(ent_owner.size());
+    for (int g = 0; g < c->G; ++g) R0[g + 1] = R0[g] + Br0 * nloc[g];
+    for (size_t e = 0; e < ent_owner.size(); ++e) {
+      pbase[e] = R0[ent_owner[e]] + ent_k[e];
+      pstride[e] = nloc[ent_owner[e]];
+    }
+    c->nloc = nloc;
+    CK(c, cudaMalloc(&c->d_pbase, std::max<size_t>(pbase.size(), 1) * sizeof(int64_t)));
+    CK(c, cudaMalloc(&c->d_pstride, std::max<size_t>(pstride.size(), 1) * sizeof(int32_t)));
+    CK(c, cudaMalloc(&c->d_psoff, ent_off.size() * sizeof(int32_t)));
+    CK(c, cudaMemcpy(c->d_pbase, pbase.data(), pbase.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+    CK(c, cudaMemcpy(c->d_pstride, pstride.data(), pstride.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+    CK(c, cudaMemcpy(c->d_psoff, ent_off.data(), ent_off.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
     CK(c, cudaMalloc(&c->d_comb_tglob, c->T_sh * sizeof(int32_t)));
     CK(c, cudaMalloc(&c->d_comb_nsh, c->T_sh * sizeof(int32_t)));
     CK(c, cudaMemcpy(c->d_comb_tglob, comb_tglob.data(), c->T_sh * sizeof(int32_t), cudaMemcpyHostToDevice));
@@ -381,7 +406,6 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     c->pslot_bytes = round_up((size_t)Br * (size_t)c->T_sh * (size_t)c->S_max * (size_t)dim * 4, 512);
     c->sym_bytes += 2 * c->pslot_bytes;
   }
-  if (c->bwd_enabled && c->has_shard) FAIL(c, EMB_ERR_ARG, "backward with row-sharded tables is not supported");
   if (c->bwd_enabled) {
     if (!choose_tiling((int64_t)dim * 4, 4, 4, &c->blanes, &c->bvb, &c->bnv) || c->bnv > 4)
       FAIL(c, EMB_ERR_ARG, "backward: unsupported fp32 row size %d bytes", dim * 4);
@@ -473,6 +497,8 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_sleep_kernel);
     cudaFuncGetAttributes(&a, emb_unpack_rows_kernel<uint4>);
     cudaFuncGetAttributes(&a, emb_unpack_rows_kernel<uint2>);
+    cudaFuncGetAttributes(&a, emb_unpack_partials_kernel<float>);
+    cudaFuncGetAttributes(&a, emb_unpack_partials_kernel<__nv_bfloat16>);
     cudaFuncGetAttributes(&a, emb_combine_kernel<float>);
     cudaFuncGetAttributes(&a, emb_combine_kernel<__nv_bfloat16>);
     cudaFuncGetAttributes(&a, emb_bwd_signal_kernel);
@@ -1057,6 +1083,10 @@ emb_status_t emb_backward(emb_ctx_t* c, const int64_t* offsets, const int64_t* i
   }
   p.dW = c->d_dW;
   const bool sorted = c->bwd_algo == 1 && c->T_r > 0;
+  if (sorted && c->has_shard) {
+    c->err = "bwd_algo 1 does not support row-sharded tables (use bwd_algo 0)";
+    return abandon(EMB_ERR_ARG);
+  }
   if (sorted) {
     emb_status_t st = sorted_workspace(c, offsets, s);
     if (st != EMB_OK) return abandon(st);
@@ -1115,6 +1145,9 @@ emb_status_t emb_finalize(emb_ctx_t* c) {
   if (c->d_comb_tglob) cudaFree(c->d_comb_tglob);
   if (c->d_tmaps) cudaFree(c->d_tmaps);
   if (c->d_comb_nsh) cudaFree(c->d_comb_nsh);
+  if (c->d_pbase) cudaFree(c->d_pbase);
+  if (c->d_pstride) cudaFree(c->d_pstride);
+  if (c->d_psoff) cudaFree(c->d_psoff);
   if (c->d_unpack_stride) cudaFree(c->d_unpack_stride);
   if (c->d_off_stage) cudaFree(c->d_off_stage);
   if (c->d_idx_stage) cudaFree(c->d_idx_stage);
@@ -1253,8 +1286,14 @@ const char* emb_last_error(const emb_ctx_t* c) { return c ? c->err.c_str() : g_i
 emb_status_t emb_baseline_splits(const emb_ctx_t* c, int64_t* send_counts, int64_t* recv_counts) {
   if (!c || !send_counts || !recv_counts) return EMB_ERR_ARG;
   if (!c->registered) return EMB_ERR_STATE;
-  if (c->has_shard) return EMB_ERR_ARG;
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
+  if (c->has_shard) {                   // fp32 partials of every local shard (incl. whole tables)
+    for (int g = 0; g < c->G; ++g) {
+      send_counts[g] = (c->bstart[g + 1] - c->bstart[g]) * c->T_r * c->d;
+      recv_counts[g] = Br * (int64_t)c->nloc[g] * c->d;
+    }
+    return EMB_OK;
+  }
   for (int g = 0; g < c->G; ++g) {
     send_counts[g] = (c->bstart[g + 1] - c->bstart[g]) * c->T_r * c->d;
     recv_counts[g] = Br * (int64_t)c->tables_of[g].size() * c->d;
@@ -1266,12 +1305,17 @@ static emb_status_t baseline_pool_impl(emb_ctx_t* c, const void* offsets, const 
                                        cudaStream_t s, void* send) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_pool before emb_register_tables");
-  if (c->has_shard) FAIL(c, EMB_ERR_ARG, "the comparison path does not support row-sharded tables");
   if (c->T_r > 0 && (!offsets || !indices || !send)) FAIL(c, EMB_ERR_ARG, "NULL buffer");
   CK(c, cudaSetDevice(c->dev));
   FwdParams p;
   fill_params(c, offsets, indices, i32, false, (char*)send, &p);
   p.check = (flags & EMB_FWD_CHECK_BOUNDS) ? 1 : 0;
+  if (c->has_shard) {                   // f3: every local shard's fp32 partial, destination-major
+    p.all_partial = 1;
+    p.part_stride = c->T_r;
+    for (int g = 0; g < c->G; ++g)
+      p.part_base[g] = (char*)send + (size_t)c->bstart[g] * (size_t)c->T_r * (size_t)c->d * 4;
+  }
   return launch_fwd(c, p, flags & EMB_FWD_CHECK_BOUNDS, s);
 }
 
@@ -1288,7 +1332,6 @@ emb_status_t emb_baseline_pool_i32(emb_ctx_t* c, const int32_t* offsets, const i
 emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, void* out) {
   if (!c) return EMB_ERR_ARG;
   if (!c->registered) FAIL(c, EMB_ERR_STATE, "emb_baseline_unpack before emb_register_tables");
-  if (c->has_shard) FAIL(c, EMB_ERR_ARG, "the comparison path does not support row-sharded tables");
   if (!recv || !out) FAIL(c, EMB_ERR_ARG, "NULL buffer");
   CK(c, cudaSetDevice(c->dev));
   const int64_t Br = c->bstart[c->rank + 1] - c->bstart[c->rank];
@@ -1296,6 +1339,16 @@ emb_status_t emb_baseline_unpack(emb_ctx_t* c, const void* recv, void* stream, v
   const int64_t rows = Br * c->T;
   int grid = (int)std::min<int64_t>((rows + (kBlock / 32) - 1) / (kBlock / 32), (int64_t)c->num_sms * 8);
   if (grid < 1) grid = 1;
+  if (c->has_shard) {                   // f3: sum the shards' partials in shard order, then pack
+    if (c->odt == EMB_F32)
+      emb_unpack_partials_kernel<float><<<grid, kBlock, 0, (cudaStream_t)stream>>>(
+          (const float*)recv, (char*)out, c->d_pbase, c->d_pstride, c->d_psoff, Br, c->T, c->d);
+    else
+      emb_unpack_partials_kernel<__nv_bfloat16><<<grid, kBlock, 0, (cudaStream_t)stream>>>(
+          (const float*)recv, (char*)out, c->d_pbase, c->d_pstride, c->d_psoff, Br, c->T, c->d);
+    CK(c, cudaGetLastError());
+    return EMB_OK;
+  }
   if (rowbytes % 16 == 0)
     emb_unpack_rows_kernel<uint4><<<grid, kBlock, 0, (cudaStream_t)stream>>>((const char*)recv, (char*)out,
                                                                            c->d_unpack_base, c->d_unpack_stride, Br,

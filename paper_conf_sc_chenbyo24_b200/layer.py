@@ -59,6 +59,7 @@ class PgasEmbedding:
         self.B = global_batch
         self.B_r = self.info["local_batch"]
         self.out_dtype = _tdt(self.info["out_dtype"])
+        self.sharded = shards is not None
         self._send = self._recv = self._out = None
 
     # ---- PGAS fused path (Listing 2) ----------------------------------------------------
@@ -74,8 +75,10 @@ class PgasEmbedding:
         if self._send is None:
             sc, rc = E.emb_baseline_splits(self.ctx)
             self._send_counts, self._recv_counts = sc, rc
-            self._send = torch.empty(max(sum(sc), 1), dtype=self.out_dtype, device=self.device)
-            self._recv = torch.empty(max(sum(rc), 1), dtype=self.out_dtype, device=self.device)
+            # f3 row-sharded tables exchange fp32 partials (combined in shard order by the unpack)
+            xdt = torch.float32 if self.sharded else self.out_dtype
+            self._send = torch.empty(max(sum(sc), 1), dtype=xdt, device=self.device)
+            self._recv = torch.empty(max(sum(rc), 1), dtype=xdt, device=self.device)
             self._out = torch.empty((self.B_r, self.T, self.dim), dtype=self.out_dtype, device=self.device)
         return self._send, self._recv, self._out
 
@@ -89,7 +92,12 @@ class PgasEmbedding:
         always_exchange: run the collective + unpack even at G = 1 (a self-exchange)."""
         send, recv, out = self._baseline_buffers()
         E.emb_baseline_pool(self.ctx, offsets, indices, send, flags, stream)
-        if (self.ctx.world_size == 1 and not always_exchange) or pool_only:
+        if pool_only:
+            return send
+        if self.ctx.world_size == 1 and not always_exchange:
+            if self.sharded:     # G = 1, row shards: no exchange, the partials still need their combine
+                E.emb_baseline_unpack(self.ctx, send, out, stream)
+                return out
             # G = 1: send already is [B][T][d]; no exchange, no unpack
             return send[: self.B_r * self.T * self.dim].view(self.B_r, self.T, self.dim)
         import torch.distributed as dist

@@ -179,3 +179,103 @@ def test_sharded_check_bounds():
                         exp[b, t] += full[t][v]
     cat = np.concatenate(got, axis=0)
     assert np.array_equal(cat, exp)
+
+
+@pytest.mark.parametrize("G", [1, 2, 3])
+def test_sharded_backward_integer_exact(G):
+    """f2 on f3 row-sharded tables: every shard owner pulls the DP ranks' dY of its table's
+    bags and scatters into ITS rows only; the expected dW of shard (t, s) is rows [lo, hi)
+    of the table-wise transpose (the oracle's emb_backward on a one-rank placement of the
+    same bags), exact on integer gradients over 2 epochs."""
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=40, B=61, T=4, dim=64, rows=500, dist="zipf")
+    shards = _shards(w, lambda t: [2, 1, 3, 2][t], lambda t, s: (t + s) % G)
+    tabs = H.np_tables(w)
+    full = [tabs[int(w.phys[t])] for t in range(w.T)]
+    dev_full = [torch.from_numpy(a).to(DEV) for a in full]
+    mine = [sorted((t, s, lo, hi) for (t, s, lo, hi, o) in shards if o == r) for r in range(G)]
+    local_w = [[dev_full[t][lo:hi] for (t, s, lo, hi) in mine[r]] for r in range(G)]
+    grp = LocalGroup(G) if G > 1 else None
+    layers = run_ranks(G, lambda r: PgasEmbedding(r, G, 0, w.rows, None, w.dim, local_w[r], w.B, w.wdtype, w.odtype,
+                                                  grp.allgather_for(r) if grp else None, {"timeout_ms": 20000},
+                                                  backward=True, shards=shards))
+    try:
+        offs, idxs = _inputs(w, 17, shards)
+        ins = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(G)]
+        starts, counts = O.split_batch(w.B, G)
+        rng = np.random.default_rng(5)
+        dW = [[torch.zeros((hi - lo, w.dim), device=DEV) for (t, s, lo, hi) in mine[r]] for r in range(G)]
+        streams = [torch.cuda.Stream() for _ in range(G)]
+        dYs = []
+        for ep in range(2):
+            dY = [rng.integers(-8, 9, size=(counts[r], w.T, w.dim)).astype(np.float32) for r in range(G)]
+            dYs.append(dY)
+            for r in range(G):
+                with torch.cuda.stream(streams[r]):
+                    layers[r].grad_slot(streams[r]).copy_(torch.from_numpy(dY[r]).to(DEV))
+                layers[r].grad_ready(streams[r])
+            for r in range(G):
+                layers[r].backward(ins[r][0], ins[r][1], dW[r], 0, streams[r], publish=False)
+            torch.cuda.synchronize()
+        errs = [layers[r].device_error() for r in range(G)]
+    finally:
+        run_ranks(G, lambda r: layers[r].close())
+    assert errs == [0] * G
+    wt = synth.make_workload("tiny", G=1, pmin=0, pmax=40, B=61, T=4, dim=64, rows=500, dist="zipf")
+    o1, x1 = synth.rank_csr(wt, 17, 0)
+    ref = None
+    for dY in dYs:
+        r_ep, _, _ = O.emb_backward(w.rows, w.dim, wt.owner, [o1], [x1], [np.concatenate(dY, 0)], w.B, 1)
+        ref = r_ep if ref is None else [a + b for a, b in zip(ref, r_ep)]
+    for r in range(G):
+        for k, (t, s, lo, hi) in enumerate(mine[r]):
+            assert np.array_equal(dW[r][k].cpu().numpy().astype(np.float64), ref[t][lo:hi]), (r, t, s)
+
+
+@pytest.mark.parametrize("G,odt", [(1, "f32"), (2, "f32"), (3, "f32"), (2, "bf16")])
+def test_sharded_comparison_path_matches_fused_bitwise(G, odt):
+    """f3 comparison path (pool every local shard's fp32 partial destination-major ->
+    all-to-all, done with copies here -> unpack summing each table's partials in shard
+    order) equals the fused PGAS path bit for bit, and both equal the sharded oracle."""
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=40, B=73, T=5, dim=64, rows=900, dist="zipf", odtype=odt)
+    shards = _shards(w, lambda t: [1, 2, 3, 1, 4][t], lambda t, s: (t + 2 * s) % G)
+    tabs = H.np_tables(w)
+    full = [tabs[int(w.phys[t])] for t in range(w.T)]
+    dev_full = [torch.from_numpy(a).to(DEV) for a in full]
+    local_w = [[dev_full[t][lo:hi] for (t, s, lo, hi, o) in sorted(shards) if o == r] for r in range(G)]
+    grp = LocalGroup(G) if G > 1 else None
+    layers = run_ranks(G, lambda r: PgasEmbedding(r, G, 0, w.rows, None, w.dim, local_w[r], w.B, w.wdtype, w.odtype,
+                                                  grp.allgather_for(r) if grp else None, {"timeout_ms": 20000},
+                                                  shards=shards))
+    try:
+        offs, idxs = _inputs(w, 29, shards)
+        ins = [(torch.from_numpy(offs[r]).to(DEV), torch.from_numpy(idxs[r]).to(DEV)) for r in range(G)]
+        streams = [torch.cuda.Stream() for _ in range(G)]
+        torch.cuda.synchronize()
+        yd = [layers[r].forward(ins[r][0], ins[r][1], 0, streams[r]) for r in range(G)]
+        torch.cuda.synchronize()
+        ys = [H.dev_out_to_np(y) for y in yd]
+        sends, splits = [], []
+        for r in range(G):
+            sc, rc = E.emb_baseline_splits(layers[r].ctx)
+            snd = torch.full((max(sum(sc), 1),), float("nan"), device=DEV)
+            E.emb_baseline_pool(layers[r].ctx, ins[r][0], ins[r][1], snd)
+            sends.append(snd)
+            splits.append((sc, rc))
+        torch.cuda.synchronize()
+        outs = []
+        for r in range(G):                                # all_to_all_single semantics, with copies
+            recv = torch.cat([sends[src][sum(splits[src][0][:r]): sum(splits[src][0][:r]) + splits[src][0][r]]
+                              for src in range(G)])
+            assert recv.numel() == sum(splits[r][1])
+            out = torch.full((layers[r].B_r, w.T, w.dim), float("nan"), device=DEV).to(layers[r].out_dtype)
+            E.emb_baseline_unpack(layers[r].ctx, recv, out)
+            torch.cuda.synchronize()
+            outs.append(H.dev_out_to_np(out))
+        errs = [layers[r].device_error() for r in range(G)]
+    finally:
+        run_ranks(G, lambda r: layers[r].close())
+    assert errs == [0] * G
+    ref = O.emb_forward_sharded(full, shards, offs, idxs, w.B, w.G, out_dtype=w.odtype)
+    for r in range(G):
+        assert np.array_equal(H.bits(outs[r]), H.bits(ys[r])), r
+        assert np.array_equal(H.bits(outs[r]), H.bits(ref[r])), r
