@@ -55,6 +55,13 @@ def test_bench_two_ranks_one_gpu():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
            "127.0.0.1", "--master-port", "29561", "bench.py", "--gpus", "2", "--steps", "5", "--warmup", "3",
            "--config", "tiny", "--backend", "gloo", "--same-device", "--repeats", "3"]
+    # f3 at N = 2: shards spread over both ranks, fused path and comparison path (fp32 partials)
+    rs = subprocess.run(cmd[:-2] + ["--repeats", "2", "--shards", "2", "--no-cpu-baseline", "--no-e2e"], cwd=ROOT,
+                        capture_output=True, text=True, timeout=900)
+    assert rs.returncode == 0, rs.stderr[-3000:]
+    ds = _last_json(rs.stdout)
+    assert ds["config"]["row_shards_per_table"] == 2 and ds["value"] > 0
+    assert ds["comparison_nccl_path"]["breakdown"]["exchange_phase_ms"] >= 0
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-3000:]
     d = _last_json(r.stdout)
