@@ -115,7 +115,9 @@ emb_status_t emb_init(int rank, int world_size, int cuda_device, emb_allgather_f
  *   weight_dtype / out_dtype : EMB_F32 or EMB_BF16 (accumulation is always fp32, C5;
  *                bf16 output is RNE-rounded once, C6)
  *   global_batch: B >= world_size; rank r's mini-batch is the contiguous block
- *                [s_r, s_r + B_r), first B mod G ranks one extra sample (C8)
+ *                [s_r, s_r + B_r), first B mod G ranks one extra sample (C8);
+ *                (T + 1) * B <= 2^31 - 1, T counting every row shard (the fused
+ *                kernel's 32-bit work counter)
  *   local_weights[T_r] : device pointers of this rank's tables in ascending global id,
  *                row-major [M_t][d], 16-byte aligned; zero-copy: the caller keeps them
  *                alive until emb_finalize.

@@ -266,6 +266,12 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
   if (out_dtype != EMB_F32 && out_dtype != EMB_BF16) FAIL(c, EMB_ERR_ARG, "bad out dtype");
   if (global_batch < c->G) FAIL(c, EMB_ERR_ARG, "global_batch %lld < world_size %d", (long long)global_batch, c->G);
   if (dim < 1) FAIL(c, EMB_ERR_ARG, "dim %d < 1", dim);
+  // the forward's work counter is 32-bit: (local shards + 1) x B bags bound the chunks
+  int64_t nsh = 0;
+  for (int t = 0; t < num_tables; ++t) nsh += num_shards[t] > 0 ? num_shards[t] : 0;
+  if ((nsh + 1) * global_batch > (int64_t)INT32_MAX)
+    FAIL(c, EMB_ERR_ARG, "(table shards + 1) * global_batch = %lld exceeds 2^31 - 1",
+         (long long)(nsh + 1) * (long long)global_batch);
   const size_t wsz = esize(weight_dtype), osz = esize(out_dtype);
   int lanes, vb, nv;
   if (!choose_tiling((int64_t)dim * wsz, wsz, osz, &lanes, &vb, &nv))

@@ -373,6 +373,10 @@ def test_api_errors():
             E.emb_register_tables(ctx, [10], [1], 4, "f32", "f32", 4, [w])  # owner out of range
         with pytest.raises(E.EmbError):
             E.emb_set_option(ctx, "nope", 1)
+        w4 = torch.zeros((10, 4), device=DEV)
+        with pytest.raises(E.EmbError) as ei:     # (T + 1) * B > 2^31 - 1: 32-bit work counter
+            E.emb_register_tables(ctx, [10], [0], 4, "f32", "f32", 2 ** 30, [w4])
+        assert ei.value.status == 1 and "2^31" in str(ei.value)
     finally:
         E.emb_finalize(ctx)
 
