@@ -669,7 +669,7 @@ def main():
 
         def fwd_u(s):
             layer.forward(ub[s % 2][0], ub[s % 2][1], 0, stream)
-        ms_u, _ = H.timed(fwd_u, max(args.steps // 2, 3), what="uniform_control")
+        ms_u, _ = H.timed(fwd_u, args.steps, what="uniform_control")
         t_roof_u = H.allreduce_max(max(cb_u / (peak * 1e9), t_nvl))
         hb_u = algorithmic_bytes(wu, float(np.mean(nnz_u)), nbags, ib)
         extra["uniform_control"] = {"ms_per_step": ms_u, "value": w.B / (ms_u * 1e-3),
@@ -693,7 +693,10 @@ def main():
             return f
         for s in range(3):
             run_b(False)(s)
-        k_b = max(args.steps // 2, 3)
+        # same step count as the fused path: sustained runs slow down under the power cap
+        # (weak zipf, one B200: 0.667 ms/step over 50 steps, 0.685 over 100, 0.722 over 200,
+        # identical for both paths), so unequal counts would bias pgas_speedup
+        k_b = args.steps
         ms_b, _ = H.timed(run_b(False), k_b, what="nccl_path")
         cmp = {"ms_per_step": ms_b, "value": w.B / (ms_b * 1e-3), "pgas_speedup": ms_b / ms}
         if N == 1:
