@@ -31,7 +31,8 @@ struct SortParams {
   const int64_t* rowbase;      // [T_r + 1] global row base of each local table (device)
   const TableDesc* tables;     // [T_r] (global id)
   uint32_t* cnt;               // [R] counts -> exclusive starts -> ends
-  uint2* pairs;                // [cap] {dY row code, global row g}
+  uint32_t* ecode;             // [cap] dY row code of each entry (gen output; sorted: reduce input)
+  uint32_t* erow;              // [cap] global dW row g of each entry (the sort key)
   uint32_t* bsum;              // [nblk] scan tile sums
   float* const* dW;            // [T_r] fp32 [M_t][d]
   const char* gsrc[kMaxG];     // per DP rank: its grad slot of this epoch, [B_dst][T][d] fp32
@@ -43,15 +44,17 @@ struct SortParams {
   int32_t T, T_r, d, G, rank, lanes, chunk_rows;
   uint32_t epoch;
   // bwd_algo 3 (LSD radix sort): ping-pong entry buffers, per-(digit, tile) histogram
-  const uint2* rin;
-  uint2* rout;
+  const uint32_t* rin_c;       // this pass's input entries (codes, rows) ...
+  const uint32_t* rin_g;
+  uint32_t* rout_c;            // ... and output
+  uint32_t* rout_g;
   uint32_t* ghist;             // [256][nblk_r], digit-major
   int64_t nblk_r;
   int32_t shift;
 };
 
 constexpr int kScanTile = 4096;    // counters per scan tile (256 threads x 16)
-constexpr int kSortTask = 256;     // sorted entries per warp task in reduce
+constexpr int kSortTask = 512;     // sorted entries per warp task in reduce (multiple of 128)
 
 __device__ __forceinline__ int64_t sort_nnz(const SortParams& p) {
   return __ldg(p.offsets + (int64_t)p.T_r * p.B);
@@ -192,7 +195,8 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_gen_kernel(const __grid_con
       int dst = 0;
       while (b >= p.bstart[dst + 1]) ++dst;
       const uint32_t code = ((uint32_t)dst << 28) | (uint32_t)((b - p.bstart[dst]) * p.T + tglob);
-      p.pairs[j] = make_uint2(code, (uint32_t)(rb + ld_stream_i64(p.indices + j)));
+      p.ecode[j] = code;
+      p.erow[j] = (uint32_t)(rb + ld_stream_i64(p.indices + j));
     }
     __syncwarp();
   }
@@ -211,7 +215,7 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_up_kernel(const __grid_cons
 #pragma unroll 4
     for (int i = 0; i < kRTile / kBlock; ++i) {
       const int64_t idx = base + (int64_t)i * kBlock + threadIdx.x;
-      if (idx < nnz) atomicAdd(hist + ((p.rin[idx].y >> p.shift) & (kRBins - 1)), 1u);
+      if (idx < nnz) atomicAdd(hist + ((p.rin_g[idx] >> p.shift) & (kRBins - 1)), 1u);
     }
   }
   __syncthreads();
@@ -248,7 +252,7 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_down_kernel(const __grid_co
 #pragma unroll
   for (int i = 0; i < KI; ++i) {
     const int64_t idx = wbase + 32 * i + lane;
-    e[i] = idx < nnz ? p.rin[idx] : make_uint2(0u, 0xffffffffu);
+    e[i] = idx < nnz ? make_uint2(p.rin_c[idx], p.rin_g[idx]) : make_uint2(0u, 0xffffffffu);
   }
 #pragma unroll
   for (int i = 0; i < KI; ++i) {
@@ -299,37 +303,83 @@ __global__ void __launch_bounds__(kBlock) emb_bradix_down_kernel(const __grid_co
   for (int k = threadIdx.x; k < cnt; k += kBlock) {      // digit runs leave contiguously
     const uint2 v = stage[k];
     const uint32_t d = (v.y >> p.shift) & (kRBins - 1);
-    p.rout[gofs[d] + (uint32_t)k - lstart[d]] = v;
+    const uint32_t o = gofs[d] + (uint32_t)k - lstart[d];
+    p.rout_c[o] = v.x;
+    p.rout_g[o] = v.y;
   }
 }
 
-// 5. segmented gather-sum of the sorted entries + one red.add per run of equal rows
-template <int VB, int NV>
-__global__ void __launch_bounds__(kBlock) emb_bsort_reduce_kernel(const __grid_constant__ SortParams p) {
+// 5. segmented gather-sum of the sorted entries + one red.add per run of equal rows.
+// A warp claims tasks of kSortTask consecutive sorted entries; the next task's codes and
+// rows are copied into the warp's shared-memory double buffer (cp.async, 16 B per lane)
+// while the current one is summed, so no entry load sits on the critical path.  Per group
+// of UR entries one broadcast LDS.128 yields the 4 dY row codes (issue) and one the 4 dW
+// rows (consume) -- no per-entry SHFL; dY vectors are gathered in a software pipeline of
+// NGRP groups (two in flight while one is consumed for 512-B rows, as in the forward) and
+// summed with packed FADD2; a run's sum goes to dW_t[x] with one red.add per lane vector
+// when the run ends (runs crossing a task boundary add one partial per task).
+template <int VB, int NV, int NGRP = 2, int MB = 1, bool MULTI = true>
+__global__ void __launch_bounds__(kBlock, MB) emb_bsort_reduce_kernel(const __grid_constant__ SortParams p) {
   constexpr int W = VB / 4;
-  constexpr int UR = 4;                                   // rows per pipeline group
+  constexpr int UR = 4;                                   // entries per pipeline group
+  static_assert(NGRP == 2 || NGRP == 3, "groups of row vectors in registers");
+  constexpr int S = kSortTask;
+  static_assert(S % (32 * 4) == 0, "a task is whole 16-B pieces per lane");
+  constexpr int kPad = (NGRP + 1) * UR;                   // codes read ahead past a task's end
+  constexpr uint32_t kCodeB = (S + kPad) * 4u;            // codes + zero padding read by issue-ahead
+  constexpr uint32_t kBufB = kCodeB + S * 4u;             // one buffer: codes | rows
   extern __shared__ __align__(16) int64_t bs_smem[];
   int64_t* rb = bs_smem;                                  // [T_r + 1] row bases
-  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) rb[i] = __ldg(p.rowbase + i);
   const int lane = threadIdx.x & 31;
   const bool active = lane < p.lanes;
-  const int64_t rowbytes = (int64_t)p.d * 4;
+  const uint32_t rowbytes = (uint32_t)p.d * 4u;
+  // per-warp entry double buffer after the row bases
+  const uint32_t ebase = (((uint32_t)__cvta_generic_to_shared(bs_smem) + (uint32_t)(p.T_r + 1) * 8u + 15u) & ~15u) +
+                         (threadIdx.x >> 5) * (2u * kBufB);
+  for (int i = threadIdx.x; i <= p.T_r; i += blockDim.x) rb[i] = __ldg(p.rowbase + i);
+  if (lane < kPad)                                        // codes past a task's end: row 0 of rank 0
+    for (uint32_t b = 0; b < 2; ++b)
+      asm volatile("st.shared.u32 [%0], %1;" ::"r"(ebase + b * kBufB + (S + lane) * 4u), "r"(0u) : "memory");
   if (threadIdx.x == 0 && p.G > 1) wait_flags_geq(p.my_ready, p.G, p.rank, p.epoch, p.timeout_ns, &p.ctrl->err);
   __syncthreads();
+  const char* g0 = p.gsrc[0] + lane * VB;                 // !MULTI: every code is a row of rank 0's slot
   const int64_t nnz = sort_nnz(p);
   if (nnz <= p.cap) {
-    const int64_t ntask = (nnz + kSortTask - 1) / kSortTask;
+    const int64_t ntask = (nnz + S - 1) / S;
+    // stage task c's entries into buffer `buf` (the entry arrays hold >= nnz + S slots, so a
+    // task's last piece never reads past them; entries past nnz are never consumed)
+    auto stage = [&](int64_t c, uint32_t buf) {
+      const uint32_t sb = ebase + buf * kBufB;
+#pragma unroll
+      for (int k = 0; k < S / 128; ++k) {
+        const int64_t e = c * S + (int64_t)(k * 32 + lane) * 4;
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sb + (uint32_t)(k * 32 + lane) * 16u),
+                     "l"(p.ecode + e) : "memory");
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sb + kCodeB + (uint32_t)(k * 32 + lane) * 16u),
+                     "l"(p.erow + e) : "memory");
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    };
     unsigned c_next = 0;
     if (lane == 0) c_next = atomicAdd(&p.ctrl->bwork, 1u);
-    for (;;) {
-      const unsigned c = __shfl_sync(kFull, c_next, 0);
-      if ((int64_t)c >= ntask) break;
+    int64_t c = __shfl_sync(kFull, c_next, 0);
+    if (c < ntask) stage(c, 0);
+    uint32_t buf = 0;
+    while (c < ntask) {
       if (lane == 0) c_next = atomicAdd(&p.ctrl->bwork, 1u);
-      const int64_t e0 = (int64_t)c * kSortTask, e1 = min(nnz, e0 + kSortTask);
-      const int n = (int)(e1 - e0);
-      // this task's entries, one per lane per batch of 32
-      uint2 ent = lane < n ? p.pairs[e0 + lane] : make_uint2(0u, 0xffffffffu);
-      uint32_t cur = __shfl_sync(kFull, ent.y, 0);        // row of the current run
+      const int64_t cn = __shfl_sync(kFull, c_next, 0);
+      if (cn < ntask) stage(cn, buf ^ 1u);                // next task's entries in flight
+      else asm volatile("cp.async.commit_group;" ::: "memory");
+      asm volatile("cp.async.wait_group 1;" ::: "memory");   // this task's entries landed
+      __syncwarp();
+      const uint32_t sc = ebase + buf * kBufB;
+      const int n = (int)min((int64_t)S, nnz - c * S);
+      if (n < S) {                                        // the list's last task: codes past n -> 0
+        for (int k = n + lane; k < S; k += 32) asm volatile("st.shared.u32 [%0], %1;" ::"r"(sc + 4u * k), "r"(0u) : "memory");
+        __syncwarp();
+      }
+      uint32_t cur;
+      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(cur) : "r"(sc + kCodeB) : "memory");
       int t = 0;
       {
         int lo = 0, hi = p.T_r - 1;
@@ -346,8 +396,8 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_reduce_kernel(const __grid_c
       auto emit = [&]() {                                 // run of row `cur` -> dW_t[x]
         while ((int64_t)cur >= rb[t + 1]) ++t;
         if (active) {
-          float* dwt = reinterpret_cast<float*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t)));
-          char* rp = reinterpret_cast<char*>(dwt) + ((int64_t)cur - rb[t]) * rowbytes + lane * VB;
+          char* dwt = reinterpret_cast<char*>(__ldg(reinterpret_cast<const unsigned long long*>(p.dW + t)));
+          char* rp = dwt + (int64_t)((int64_t)cur - rb[t]) * rowbytes + lane * VB;
 #pragma unroll
           for (int v = 0; v < NV; ++v) {
             uint32_t u[W];
@@ -359,53 +409,86 @@ __global__ void __launch_bounds__(kBlock) emb_bsort_reduce_kernel(const __grid_c
 #pragma unroll
         for (int i = 0; i < NV * W; ++i) acc[i] = 0.0f;
       };
-      auto gaddr = [&](uint32_t code) -> const char* {
-        return p.gsrc[code >> 28] + (int64_t)(code & 0x0fffffffu) * rowbytes + lane * VB;
+      auto add_row = [&](const uint32_t (&r)[NV][W]) {
+        if (active) {
+#pragma unroll
+          for (int v = 0; v < NV; ++v) Widen<float, VB>::add(acc + v * W, r[v]);
+        }
       };
-      uint32_t bufA[UR][NV][W], bufB[UR][NV][W];
-      uint32_t gA[UR], gB[UR];
-      auto issue = [&](uint32_t (&buf)[UR][NV][W], uint32_t (&gg)[UR], const uint2& e, int j0, int jn) {
+      // the UR entries whose codes start at shared address qa: their dY vectors in flight
+      // (positions past the task read code 0 -- a valid row, loaded and never added)
+      auto issue = [&](uint32_t (&bf)[UR][NV][W], uint32_t qa) {
+        uint32_t code[UR];
+        asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(code[0]), "=r"(code[1]), "=r"(code[2]), "=r"(code[3])
+                     : "r"(qa) : "memory");
 #pragma unroll
         for (int u = 0; u < UR; ++u) {
-          const int j = j0 + u;
-          const uint32_t code = __shfl_sync(kFull, e.x, j & 31);
-          gg[u] = __shfl_sync(kFull, e.y, j & 31);
-          if (j < jn && active) {
-            const char* a = gaddr(code);
+          if (active) {
+            const char* a = MULTI ? p.gsrc[code[u] >> 28] + lane * VB : g0;
+            a = row_addr(a, MULTI ? (code[u] & 0x0fffffffu) : code[u], rowbytes);
 #pragma unroll
-            for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, buf[u][v]);
+            for (int v = 0; v < NV; ++v) ld_vec_relaxed<VB>(a + v * 32 * VB, bf[u][v]);
           }
         }
       };
-      auto consume = [&](const uint32_t (&buf)[UR][NV][W], const uint32_t (&gg)[UR], int j0, int jn) {
+      auto consume = [&](const bool PRED, const uint32_t (&bf)[UR][NV][W], uint32_t qa, int q) {
+        uint32_t g[UR];
+        asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(g[0]), "=r"(g[1]), "=r"(g[2]), "=r"(g[3])
+                     : "r"(qa + kCodeB) : "memory");
+        if (!PRED && g[UR - 1] == cur) {                  // sorted: the whole group continues the run
+#pragma unroll
+          for (int u = 0; u < UR; ++u) add_row(bf[u]);
+          return;
+        }
 #pragma unroll
         for (int u = 0; u < UR; ++u) {
-          if (j0 + u < jn) {
-            if (gg[u] != cur) {
+          if (!PRED || q + u < n) {
+            if (g[u] != cur) {
               emit();
-              cur = gg[u];
+              cur = g[u];
             }
-#pragma unroll
-            for (int v = 0; v < NV; ++v)
-#pragma unroll
-              for (int i = 0; i < W; ++i) acc[v * W + i] += __uint_as_float(buf[u][v][i]);
+            add_row(bf[u]);
           }
         }
       };
-      for (int base = 0; base < n; base += 32) {
-        const int jn = min(32, n - base);
-        if (base > 0) ent = (base + lane < n) ? p.pairs[e0 + base + lane] : make_uint2(0u, 0xffffffffu);
-        issue(bufA, gA, ent, 0, jn);
+      constexpr uint32_t kG = UR * 4u;                    // bytes of one group's codes
+      if constexpr (NGRP == 3) {
+        uint32_t A[UR][NV][W], Bv[UR][NV][W], C[UR][NV][W];
+        issue(A, sc);
+        issue(Bv, sc + kG);
+        uint32_t qa = sc;
 #pragma unroll 1
-        for (int j = 0; j < jn; j += 2 * UR) {
-          issue(bufB, gB, ent, j + UR, jn);
-          consume(bufA, gA, j, jn);
-          if (j + 2 * UR < jn) issue(bufA, gA, ent, j + 2 * UR, jn);
-          consume(bufB, gB, j + UR, jn);
+        for (int q = 0; q < n; q += 3 * UR, qa += 3 * kG) {
+          issue(C, qa + 2 * kG);
+          if (q + UR > n) { consume(true, A, qa, q); break; }
+          consume(false, A, qa, q);
+          issue(A, qa + 3 * kG);
+          if (q + 2 * UR > n) { consume(true, Bv, qa + kG, q + UR); break; }
+          consume(false, Bv, qa + kG, q + UR);
+          issue(Bv, qa + 4 * kG);
+          if (q + 3 * UR > n) { consume(true, C, qa + 2 * kG, q + 2 * UR); break; }
+          consume(false, C, qa + 2 * kG, q + 2 * UR);
+        }
+      } else {
+        uint32_t A[UR][NV][W], Bv[UR][NV][W];
+        issue(A, sc);
+        uint32_t qa = sc;
+#pragma unroll 1
+        for (int q = 0; q < n; q += 2 * UR, qa += 2 * kG) {
+          issue(Bv, qa + kG);
+          if (q + UR > n) { consume(true, A, qa, q); break; }
+          consume(false, A, qa, q);
+          issue(A, qa + 2 * kG);
+          if (q + 2 * UR > n) { consume(true, Bv, qa + kG, q + UR); break; }
+          consume(false, Bv, qa + kG, q + UR);
         }
       }
       emit();                                             // the task's last run
+      __syncwarp();                                       // buffer `buf` is restaged two tasks on
+      buf ^= 1u;
+      c = cn;
     }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
   }
   // completion: every CTA's reads of peer slots are done before the last CTA tells the
   // peers their slots may be refilled

@@ -140,8 +140,9 @@ struct emb_ctx {
   int bwd_algo = 0;                // 0: atomic scatter per bag slice; 1: radix sort + segmented sum
   int64_t bs_cap = 0, bs_R = 0;    // bwd_algo 1 workspace: entries, local rows
   int64_t* d_rowbase = nullptr;
-  uint2* d_pairs = nullptr;
-  uint2* d_pairs_b = nullptr;      // radix-sort ping-pong buffer
+  uint32_t* d_pairs = nullptr;     // entries SoA: codes [bs_stride] then rows [bs_stride]
+  uint32_t* d_pairs_b = nullptr;   // radix-sort ping-pong buffer (same layout)
+  int64_t bs_stride = 0;           // entries per array: cap + one reduce task, 32-aligned
   uint32_t* d_ghist = nullptr;     // [512][tiles] digit histograms
   uint32_t* d_rbsum = nullptr;
   int64_t rs_nblk = 0;
@@ -521,10 +522,14 @@ static emb_status_t register_impl(emb_ctx_t* c, int32_t num_tables, const int64_
     cudaFuncGetAttributes(&a, emb_bradix_gen_kernel);
     cudaFuncGetAttributes(&a, emb_bradix_up_kernel);
     cudaFuncGetAttributes(&a, emb_bradix_down_kernel);
-    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1>);
-    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1>);
-    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2>);
-    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 4>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1, 2, 1, false>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1, 2, 4, false>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2, 2, 1, false>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 4, 2, 1, false>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<8, 1, 2, 1, true>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 1, 2, 4, true>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 2, 2, 1, true>);
+    cudaFuncGetAttributes(&a, emb_bsort_reduce_kernel<16, 4, 2, 1, true>);
     cudaGetLastError();
   }
   return EMB_OK;
@@ -950,8 +955,9 @@ static emb_status_t sorted_workspace(emb_ctx_t* c, const int64_t* offsets, cudaS
     }
     c->rs_nblk = (c->bs_cap + kRTile - 1) / kRTile;
     const int64_t nh = (int64_t)kRBins * c->rs_nblk;
-    CK(c, cudaMalloc(&c->d_pairs, (size_t)c->bs_cap * sizeof(uint2)));
-    CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_cap * sizeof(uint2)));
+    c->bs_stride = (c->bs_cap + kSortTask + 31) / 32 * 32;   // a reduce task's staging never reads past
+    CK(c, cudaMalloc(&c->d_pairs, (size_t)c->bs_stride * 2 * sizeof(uint32_t)));
+    CK(c, cudaMalloc(&c->d_pairs_b, (size_t)c->bs_stride * 2 * sizeof(uint32_t)));
     CK(c, cudaMalloc(&c->d_ghist, (size_t)nh * sizeof(uint32_t)));
     CK(c, cudaMalloc(&c->d_rbsum, (size_t)((nh + kScanTile - 1) / kScanTile) * sizeof(uint32_t)));
   }
@@ -970,7 +976,8 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   q.indices = indices;
   q.rowbase = c->d_rowbase;
   q.tables = c->d_tables;
-  q.pairs = c->d_pairs;
+  q.ecode = c->d_pairs;
+  q.erow = c->d_pairs + c->bs_stride;
   q.dW = bp.dW;
   for (int g = 0; g < kMaxG; ++g) {
     q.gsrc[g] = bp.gsrc[g];
@@ -991,7 +998,6 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   q.lanes = c->blanes;
   q.chunk_rows = bp.chunk_rows;
   q.epoch = bp.epoch;
-  const size_t tsm = (size_t)(c->T_r + 1) * 2 * sizeof(int64_t);
   const int grid = c->num_sms * 8;
   emb_bradix_gen_kernel<<<grid, kBlock, 0, s>>>(q);
   int bits = 1;
@@ -999,8 +1005,8 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   const int passes = (bits + kRBits - 1) / kRBits;
   const int64_t nh = (int64_t)kRBins * c->rs_nblk, nb2 = (nh + kScanTile - 1) / kScanTile;
   const size_t dsm = (size_t)(2 * kRTile + (2 + kBlock / 32) * kRBins) * sizeof(uint32_t);
-  uint2* in = c->d_pairs;
-  uint2* out = c->d_pairs_b;
+  uint32_t* in = c->d_pairs;
+  uint32_t* out = c->d_pairs_b;
   q.ghist = c->d_ghist;
   q.nblk_r = c->rs_nblk;
   SortParams qs = q;                                    // the scan runs over the histograms
@@ -1008,8 +1014,10 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
   qs.R = nh;
   qs.bsum = c->d_rbsum;
   for (int ps = 0; ps < passes; ++ps) {
-    q.rin = in;
-    q.rout = out;
+    q.rin_c = in;
+    q.rin_g = in + c->bs_stride;
+    q.rout_c = out;
+    q.rout_g = out + c->bs_stride;
     q.shift = kRBits * ps;
     emb_bradix_up_kernel<<<(unsigned)c->rs_nblk, kBlock, 0, s>>>(q);
     emb_bsort_scan_sum_kernel<<<(unsigned)nb2, kBlock, 0, s>>>(qs);
@@ -1018,15 +1026,20 @@ static emb_status_t backward_sorted(emb_ctx_t* c, const BwdParams& bp, const int
     emb_bradix_down_kernel<<<(unsigned)c->rs_nblk, kBlock, dsm, s>>>(q);
     std::swap(in, out);
   }
-  q.pairs = in;                                         // sorted by row
+  q.ecode = in;                                         // sorted by row
+  q.erow = in + c->bs_stride;
   void (*k)(SortParams) = nullptr;
-  if (c->bvb == 8) k = emb_bsort_reduce_kernel<8, 1>;
-  else if (c->bnv == 2) k = emb_bsort_reduce_kernel<16, 2>;
-  else if (c->bnv == 4) k = emb_bsort_reduce_kernel<16, 4>;
-  else k = emb_bsort_reduce_kernel<16, 1>;
+  const bool multi = c->G > 1;
+  if (c->bvb == 8) k = multi ? emb_bsort_reduce_kernel<8, 1, 2, 1, true> : emb_bsort_reduce_kernel<8, 1, 2, 1, false>;
+  else if (c->bnv == 2) k = multi ? emb_bsort_reduce_kernel<16, 2, 2, 1, true> : emb_bsort_reduce_kernel<16, 2, 2, 1, false>;
+  else if (c->bnv == 4) k = multi ? emb_bsort_reduce_kernel<16, 4, 2, 1, true> : emb_bsort_reduce_kernel<16, 4, 2, 1, false>;
+  else k = multi ? emb_bsort_reduce_kernel<16, 1, 2, 4, true> : emb_bsort_reduce_kernel<16, 1, 2, 4, false>;
+  // row bases + per-warp double buffer of one task's codes and rows
+  const size_t rsm = ((size_t)(c->T_r + 1) * 8 + 15) / 16 * 16 + (size_t)(kBlock / 32) * 2 * (2 * kSortTask + 16) * 4;
+  CK(c, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rsm));
   int per_sm = 0;
-  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, tsm / 2));
-  k<<<c->num_sms * std::max(per_sm, 1), kBlock, tsm / 2, s>>>(q);
+  CK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kBlock, rsm));
+  k<<<c->num_sms * std::max(per_sm, 1), kBlock, rsm, s>>>(q);
   CK(c, cudaGetLastError());
   return EMB_OK;
 }
