@@ -659,6 +659,7 @@ static emb_status_t fill_params(emb_ctx_t* c, const void* offsets, const void* i
     for (int g = 0; g < c->G; ++g)  // send = [G][B_dst][T_r][d]: block of dst starts at s_dst*T_r rows
       p->out_base[g] = send + (size_t)c->bstart[g] * (size_t)c->T_r * (size_t)c->d * osz;
   }
+  p->ostep = p->rowstride * (int64_t)c->d * (int64_t)osz;
   p->epoch = (uint32_t)c->epoch;
   p->trace = c->trace;
   p->trace_cap = c->trace_cap;
