@@ -171,3 +171,18 @@ def test_bwd_sorted_capacity_error():
         assert L.device_error(clear=True) & 0x4
     finally:
         L.close()
+
+
+@pytest.mark.parametrize("G,dim,algo", [(1, 128, 1), (2, 128, 1), (1, 64, 1), (1, 128, 0)])
+def test_bwd_medium_many_tasks_integer_exact(G, dim, algo):
+    """a size where bwd_algo 1's sorted list spans hundreds of 512-entry reduce tasks, zipf-hot
+    rows' runs cross task boundaries (one partial red.add per task) and the last task is ragged;
+    also the radix passes' multi-tile histograms and the atomic default at the same size: exact
+    on integer gradients against the oracle's transpose"""
+    w = synth.make_workload("tiny", G=G, pmin=0, pmax=90, B=3001, T=6, dim=dim, rows=20000, dist="zipf")
+    dY = _dY(w, 41, integer=True)
+    got, offs, idxs = _run_bwd(w, dY, 42, opts={"bwd_algo": algo})
+    assert sum(int(o[-1]) for o in offs) > 100 * 512
+    ref, _, _ = O.emb_backward(w.rows, w.dim, w.owner, offs, idxs, dY, w.B, w.G)
+    for t in range(w.T):
+        assert np.array_equal(got[t].astype(np.float64), ref[t]), t
