@@ -30,9 +30,13 @@ constexpr int BATCH = 128;   // ids staged per warp per batch
 __device__ __forceinline__ void ldg4(const char* p, float4& v) {
   asm volatile("ld.global.nc.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
 }
+// L1::no_allocate: does a load that bypasses L1 allocation skip the fill wavefronts?
+__device__ __forceinline__ void ldg4_na(const char* p, float4& v) {
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+}
 
 // ids of this warp's batch -> shared (coalesced LDG + STS), then the gather
-template <int WARPS>
+template <int WARPS, bool NA = false>
 __global__ void __launch_bounds__(WARPS * 32) bcast_kernel(const char* __restrict__ table, const uint32_t* __restrict__ ids,
                                                            long n, float* out) {
   __shared__ __align__(16) uint32_t sid[WARPS][BATCH];
@@ -52,7 +56,10 @@ __global__ void __launch_bounds__(WARPS * 32) bcast_kernel(const char* __restric
       uint32_t x[4];
       asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(x[0]), "=r"(x[1]), "=r"(x[2]), "=r"(x[3]) : "r"(sb + 4 * j) : "memory");
 #pragma unroll
-      for (int u = 0; u < 4; ++u) ldg4(base + (size_t)x[u] * ROWB, r[u]);
+      for (int u = 0; u < 4; ++u) {
+        if (NA) ldg4_na(base + (size_t)x[u] * ROWB, r[u]);
+        else ldg4(base + (size_t)x[u] * ROWB, r[u]);
+      }
     };
     auto consume = [&](float4 (&r)[4]) {
 #pragma unroll
@@ -169,6 +176,9 @@ int main(int argc, char** argv) {
     float ms = time_it([&] { bcast_kernel<8><<<grid, 256>>>(table, ids, n, out); });
     CK(cudaGetLastError());
     printf("{\"variant\": \"bcast\", \"ctas_per_sm\": %d, \"ms\": %.4f, \"GBps\": %.1f}\n", cps, ms, bytes / (ms * 1e-3) / 1e9);
+    ms = time_it([&] { bcast_kernel<8, true><<<grid, 256>>>(table, ids, n, out); });
+    CK(cudaGetLastError());
+    printf("{\"variant\": \"bcast_no_allocate\", \"ctas_per_sm\": %d, \"ms\": %.4f, \"GBps\": %.1f}\n", cps, ms, bytes / (ms * 1e-3) / 1e9);
     ms = time_it([&] { quad_kernel<8><<<grid, 256>>>(table, ids, n, out); });
     CK(cudaGetLastError());
     printf("{\"variant\": \"quad\", \"ctas_per_sm\": %d, \"ms\": %.4f, \"GBps\": %.1f}\n", cps, ms, bytes / (ms * 1e-3) / 1e9);
