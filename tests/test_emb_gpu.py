@@ -540,3 +540,25 @@ def test_c7_ieee_special_values_bitexact(dim, wdt, odt, G):
             assert layers[r].device_error() == 0
     finally:
         _close(layers)
+
+
+@pytest.mark.parametrize("G,T", [(2, 9), (3, 13), (1, 3)])
+@pytest.mark.parametrize("opts", [{}, {"chunk_rows": 7}, {"tail_div": 16, "chunk_rows": 40}, {"stagger": 0},
+                                  {"fwd_interleave": 1}])
+def test_chunk_grid_guided_tail_and_rotation_bitexact(G, T, opts):
+    """the claim -> (table, first bag) decode: ranks with >= 4 local tables take the guided tail
+    (the last table in smaller chunks), ranks with fewer do not; destination-staggered rotation
+    of the chunk order at G > 1, with chunks crossing mini-batch boundaries; bit-exact"""
+    w = synth.make_workload("tiny", G=G, T=T, dim=64, pmin=0, pmax=30, B=301, rows=500)
+    assert G == 1 or min(len(w.local_tables(r)) for r in range(G)) >= 4
+    tabs = H.np_tables(w)
+    csr = H.np_csrs(w, 73)
+    ref = H.oracle_outputs(w, 73, tabs, csr)
+    layers = _layers(w, tabs, options=opts)
+    try:
+        got = _run(w, layers, csr)
+        for r in range(w.G):
+            _assert_exact(got[r], ref[r])
+            assert layers[r].device_error() == 0
+    finally:
+        _close(layers)
